@@ -1,0 +1,399 @@
+#!/usr/bin/env python3
+"""Benchmark of the hot path: batched variable-size LU (implicit pivoting) +
+triangular solves on B200, one process per GPU.
+
+Default workload (BASELINE.json metric, north-star target): config C3 -- 1M
+blocks per GPU with orders m ~ U{4..32}, fp64.  A *step* is one pass of the
+whole hot path over one batch: layout (a1) + size plan + GETRF (a3) + GETRS
+(a4).  Each step factors its own pristine copy of the batch (generated before
+the timed region; 3.2 GB >> 126 MB L2, so no L2 flush is needed).
+
+Multi-GPU (torchrun, NCCL): the global batch of N x 1M blocks is split by the
+contiguous cost-balanced partitioner (row a6); ranks regenerate their shard
+from the counter generator; no collective on the data path; barrier + max
+over ranks of the CUDA-event time.
+
+``--impl reference`` times the CPU oracle (the reference arm of this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (nblocks per GPU, lo, hi, dtype, description)
+    "C3": (1_000_000, 4, 32, torch.float64, "C3: 1M blocks/GPU, m ~ U{4..32}, fp64, LU + solve"),
+    "C3f32": (1_000_000, 4, 32, torch.float32, "C3: 1M blocks/GPU, m ~ U{4..32}, fp32, LU + solve"),
+    "C2": (40_000, 32, 32, torch.float64, "C2: 40,000 blocks 32x32/GPU, fp64, LU + solve"),
+    "C1": (1_000, 4, 16, torch.float64, "C1: 1,000 blocks m ~ U{4..16}, fp64 (latency case, L2-resident)"),
+}
+
+
+def esize(dt):
+    return 8 if dt == torch.float64 else 4
+
+
+def algorithmic_bytes(sizes: np.ndarray, dt) -> tuple[int, int]:
+    """GETRF 2 s m^2 + 4m + 4 + 16; GETRS s m^2 + 4m + 2 s m + 16."""
+    s = esize(dt)
+    m = sizes.astype(np.int64)
+    getrf = int((2 * s * m * m + 4 * m + 4 + 16).sum())
+    getrs = int((s * m * m + 4 * m + 2 * s * m + 16).sum())
+    return getrf, getrs
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks / throttle reasons during the timed region."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower() in ("active", "1", "yes"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_setup(args):
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    return ws, rank, local
+
+
+def barrier(ws):
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+def max_over_ranks(v: float, ws: int) -> float:
+    if ws == 1:
+        return v
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# --------------------------------------------------------------------------
+# CPU oracle timing (cpu_baseline leg and --impl reference)
+# --------------------------------------------------------------------------
+def oracle_sample(nb_target: int, lo: int, hi: int, dt, budget_s: float, first: int = 0):
+    """Time oracle GETRF+GETRS on the first blocks of the workload (same
+    generator), growing the sample in chunks until ~budget_s of CPU work."""
+    import bj_synth as S
+    import oracle
+    npdt = np.float64 if dt == torch.float64 else np.float32
+    chunk = 20000 if hi > 16 else 100000
+    done, t_total = 0, 0.0
+    while done < nb_target and t_total < budget_s:
+        n = min(chunk, nb_target - done)
+        sizes = S.block_sizes(n, lo, hi, first=first + done)
+        vec, val = oracle.layout(sizes, esize(dt))
+        A = S.block_values(sizes, val, first=first + done, dtype=npdt)
+        b = S.rhs_values(sizes, first=first + done, dtype=npdt)
+        t0 = time.perf_counter()
+        LU, piv, info = oracle.getrf_batch(sizes, val, vec, A)
+        oracle.getrs_batch(sizes, val, vec, LU, piv, b)
+        t_total += time.perf_counter() - t0
+        done += n
+    return done, t_total, oracle.max_threads()
+
+
+def run_reference(args, ws, rank):
+    nb, lo, hi, dt, desc = CONFIGS[args.config]
+    if rank != 0:
+        return
+    budget = max(2.0, min(20.0, 60.0 / max(args.steps + args.warmup, 1)))
+    times = []
+    blocks = 0
+    for i in range(args.warmup + args.steps):
+        done, t, cores = oracle_sample(nb, lo, hi, dt, budget)
+        if i >= args.warmup:
+            times.append(t)
+            blocks += done
+    tot = sum(times)
+    value = blocks / tot
+    line = {
+        "impl": "reference", "metric": "blocks/s (batched LU + solve)", "value": value, "unit": "blocks/s",
+        "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * tot / max(args.steps, 1), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32", "data": "synthetic",
+        "config": {"workload": desc, "sample": f"first {blocks // max(args.steps, 1)} blocks of the workload per step"},
+        "cpu_baseline": {"value": value, "unit": "blocks/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{blocks // max(args.steps, 1)} blocks per step (GETRF+GETRS)"},
+        "e2e": {"value": value, "unit": "blocks/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------
+# GPU arm
+# --------------------------------------------------------------------------
+def run_ours(args, ws, rank, local):
+    from paper_conf_icpp_anztdfq17_b200 import bj
+    nb_per, lo, hi, dt, desc = CONFIGS[args.config]
+    if args.nblocks:
+        nb_per = args.nblocks
+    nb_total = nb_per * ws
+    # --- partition (row a6): global sizes from the counter generator
+    sizes_all = bj.synth_sizes(nb_total, lo, hi)
+    sizes_h = sizes_all.cpu().numpy()
+    bounds = bj.partition(sizes_h, ws)
+    first, last = int(bounds[rank]), int(bounds[rank + 1])
+    nb = last - first
+    sizes = sizes_all[first:last].clone()
+    del sizes_all
+    my_sizes = sizes_h[first:last]
+    getrf_bytes, getrs_bytes = algorithmic_bytes(my_sizes, dt)
+
+    base = bj.new_batch(sizes, dt)
+    bj.synth_blocks(base, first=first)
+    rhs = bj.synth_rhs(base, first=first)
+    nvec = int(base.vec_off[-1].item())
+    piv = torch.empty(max(nvec, 1), dtype=torch.int32, device="cuda")
+    info = torch.empty(max(nb, 1), dtype=torch.int32, device="cuda")
+    x = torch.empty_like(rhs)
+
+    # pool of pristine copies (one per step, inputs > L2)
+    copy_bytes = base.values.numel() * esize(dt)
+    free = torch.cuda.mem_get_info()[0]
+    cap = max(1, int((free - 8e9) // max(copy_bytes, 1)))
+    pool_n = max(1, min(args.steps + args.warmup, cap, 64))
+    pool = [base.values.clone() for _ in range(pool_n)]
+
+    stream = torch.cuda.current_stream()
+
+    def one_step(values, evs=None):
+        vec = base.vec_off
+        val = base.val_off
+        if evs is not None:
+            evs[0].record(stream)
+        v2, l2 = bj.layout(sizes, dt)                       # a1 (recomputed per step)
+        plan = bj.Plan(sizes)                               # size buckets
+        batch = bj.Batch(sizes, v2, l2, values)
+        if evs is not None:
+            evs[1].record(stream)
+        bj.getrf(batch, piv, info, plan=plan)               # a3
+        if evs is not None:
+            evs[2].record(stream)
+        bj.getrs(batch, piv, rhs, x, plan=plan)             # a4
+        if evs is not None:
+            evs[3].record(stream)
+        return plan
+
+    # warm-up
+    keep = []
+    for i in range(args.warmup):
+        keep.append(one_step(pool[i % pool_n]))
+    barrier(ws)
+    for p in keep:
+        p.close()
+    keep = []
+    for i in range(min(args.warmup, pool_n)):                # restore used copies
+        pool[i].copy_(base.values)
+    barrier(ws)
+
+    # timed region(s): chunks of at most pool_n steps, restore between chunks
+    done = 0
+    t_total_ms = 0.0
+    per = []
+    bj.launch_count_reset()
+    launches = 0
+    sampler = ClockSampler(local)
+    with sampler:
+        while done < args.steps:
+            n = min(pool_n, args.steps - done)
+            evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(n)]
+            barrier(ws)
+            start = torch.cuda.Event(enable_timing=True)
+            end = torch.cuda.Event(enable_timing=True)
+            bj.launch_count_reset()
+            start.record(stream)
+            for i in range(n):
+                keep.append(one_step(pool[i], evs[i]))
+            end.record(stream)
+            launches += bj.launch_count()
+            barrier(ws)
+            t_total_ms += start.elapsed_time(end)
+            for e in evs:
+                per.append((e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[2].elapsed_time(e[3])))
+            for p in keep:
+                p.close()
+            keep = []
+            done += n
+            if done < args.steps:
+                for i in range(min(n, pool_n)):
+                    pool[i].copy_(base.values)
+    t_ms = max_over_ranks(t_total_ms, ws)
+    per = np.array(per)
+    plan_ms, getrf_ms, getrs_ms = (float(per[:, j].mean()) for j in range(3))
+    getrf_ms = max_over_ranks(getrf_ms, ws)
+    getrs_ms = max_over_ranks(getrs_ms, ws)
+    clocks = sampler.summary()
+
+    # correctness sentinel on the timed data (cheap): no zero pivots expected
+    bad = int((info[:nb] != 0).sum().item())
+
+    hbm, peak_src = load_peaks()
+    dom = "getrf" if getrf_ms >= getrs_ms else "getrs"
+    dom_bytes, dom_ms = (getrf_bytes, getrf_ms) if dom == "getrf" else (getrs_bytes, getrs_ms)
+    achieved = dom_bytes / (dom_ms * 1e-3) / 1e9
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tf):
+        traffic = json.load(open(tf)).get(f"{args.config}:{dom}")
+    step_bytes = getrf_bytes + getrs_bytes
+    ms_per_step = t_ms / args.steps
+    value = nb_total / (ms_per_step * 1e-3)
+
+    # ---- e2e: the C-ABI call with HOST buffers (bj_gesv_host), copies inside
+    e2e = None
+    if not args.no_e2e:
+        ws_obj = bj.Workspace()
+        sizes_pin = sizes.cpu().pin_memory()
+        A_pin = base.values.cpu().pin_memory()
+        b_pin = rhs.cpu().pin_memory()
+        x_pin = torch.empty_like(b_pin).pin_memory()
+        p_pin = torch.empty(max(nvec, 1), dtype=torch.int32).pin_memory()
+        i_pin = torch.empty(max(nb, 1), dtype=torch.int32).pin_memory()
+        e2e_steps = max(1, min(args.steps, 3))
+        ws_obj.gesv_host(sizes_pin, A_pin, b_pin, x_pin, p_pin, i_pin)        # warm-up
+        barrier(ws)
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for _ in range(e2e_steps):
+            ws_obj.gesv_host(sizes_pin, A_pin, b_pin, x_pin, p_pin, i_pin)
+        t1.record(stream)
+        barrier(ws)
+        e_ms = max_over_ranks(t0.elapsed_time(t1) / e2e_steps, ws)
+        h2d = sizes_pin.numel() * 4 + A_pin.numel() * esize(dt) + b_pin.numel() * esize(dt)
+        d2h = x_pin.numel() * esize(dt) + p_pin.numel() * 4 + i_pin.numel() * 4
+        e2e = {"value": nb_total / (e_ms * 1e-3), "unit": "blocks/s", "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": e_ms, "steps": e2e_steps,
+               "api": "bj_gesv_host (pinned host buffers, synchronous)"}
+        ws_obj.close()
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu:
+        done_b, t_cpu, cores = oracle_sample(nb_per, lo, hi, dt, args.cpu_budget)
+        cpu = {"value": done_b / t_cpu, "unit": "blocks/s", "cores": cores, "kind": "oracle",
+               "sample": f"first {done_b} blocks of the workload (GETRF+GETRS, OpenMP over blocks)"}
+
+    if rank == 0:
+        line = {
+            "metric": "blocks/s (batched LU + solve)", "value": value, "unit": "blocks/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32",
+            "data": "synthetic (counter-based splitmix64, generated on device)",
+            "config": {"workload": desc, "nblocks_total": nb_total, "sizes": f"U{{{lo}..{hi}}}",
+                       "step": "layout + plan + getrf + getrs", "parallelism": f"dp{ws} (contiguous cost-balanced shards)",
+                       "l2": f"inputs larger than L2: each step factors its own pristine {copy_bytes / 1e9:.2f} GB copy"},
+            "roofline": {"bound": "hbm", "kernel": f"bj_{dom}_vbatched (size-class launches)", "achieved": achieved,
+                         "peak": hbm, "unit": "GB/s", "frac": achieved / hbm, "traffic": traffic,
+                         "peak_source": peak_src, "bytes_per_launch": dom_bytes},
+            "step_hbm": {"algorithmic_bytes": step_bytes, "achieved_gbs": step_bytes / (ms_per_step * 1e-3) / 1e9,
+                         "frac": step_bytes / (ms_per_step * 1e-3) / 1e9 / hbm},
+            "breakdown_ms": {"layout_plan": plan_ms, "getrf": getrf_ms, "getrs": getrs_ms},
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
+            "nonzero_info_blocks": bad,
+        }
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
+    ap.add_argument("--nblocks", type=int, default=0, help="override blocks per GPU")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 0)
+    if args.impl == "reference":
+        # the CPU oracle arm: rank 0 alone runs it; other ranks exit without work
+        ws = int(os.environ.get("WORLD_SIZE", "1"))
+        rank = int(os.environ.get("RANK", "0"))
+        run_reference(args, ws, rank)
+        return
+    ws, rank, local = dist_setup(args)
+    run_ours(args, ws, rank, local)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -102,10 +102,11 @@ def packed_offsets(sizes: np.ndarray, elem_size: int):
 
 
 def block_values(sizes: np.ndarray, val_off: np.ndarray, first: int = 0, dtype=np.float64,
-                 kind: str = "uniform") -> np.ndarray:
+                 kind: str = "uniform", ids=None) -> np.ndarray:
     """Packed column-major blocks.  Element (r, c) of global block g has key
     g*1024 + c*32 + r.  ``kind``: "uniform" U[-1,1) (seed 2) or "int" U{-3..3}
-    (seed 7).  fp32 values are the fp64 draws rounded to nearest."""
+    (seed 7).  fp32 values are the fp64 draws rounded to nearest.  Block i has
+    global id first+i, or ids[i] when ``ids`` is given."""
     sizes = np.asarray(sizes, dtype=np.int64)
     nb = len(sizes)
     out = np.zeros(int(val_off[nb]), dtype=dtype)
@@ -119,7 +120,8 @@ def block_values(sizes: np.ndarray, val_off: np.ndarray, first: int = 0, dtype=n
     m = sizes[blk]
     r = e % np.maximum(m, 1)
     c = e // np.maximum(m, 1)
-    key = (blk + first).astype(np.uint64) * np.uint64(BLOCK_KEY_STRIDE) + \
+    gid = (blk + first) if ids is None else np.asarray(ids, dtype=np.int64)[blk]
+    key = gid.astype(np.uint64) * np.uint64(BLOCK_KEY_STRIDE) + \
         (c * VEC_KEY_STRIDE + r).astype(np.uint64)
     if kind == "uniform":
         v = uniform_pm1(SEED_VALUES, key)
@@ -131,14 +133,15 @@ def block_values(sizes: np.ndarray, val_off: np.ndarray, first: int = 0, dtype=n
     return out
 
 
-def rhs_values(sizes: np.ndarray, first: int = 0, dtype=np.float64) -> np.ndarray:
+def rhs_values(sizes: np.ndarray, first: int = 0, dtype=np.float64, ids=None) -> np.ndarray:
     """Packed right-hand sides; element r of global block g has key g*32 + r."""
     sizes = np.asarray(sizes, dtype=np.int64)
     nb = len(sizes)
     blk = np.repeat(np.arange(nb, dtype=np.int64), sizes)
     start = np.repeat(np.cumsum(sizes) - sizes, sizes)
     r = np.arange(int(sizes.sum()), dtype=np.int64) - start
-    key = (blk + first).astype(np.uint64) * np.uint64(VEC_KEY_STRIDE) + r.astype(np.uint64)
+    gid = (blk + first) if ids is None else np.asarray(ids, dtype=np.int64)[blk]
+    key = gid.astype(np.uint64) * np.uint64(VEC_KEY_STRIDE) + r.astype(np.uint64)
     return uniform_pm1(SEED_RHS, key).astype(dtype)
 
 

@@ -1,0 +1,211 @@
+/*
+ * bj.h -- C ABI of the B200-native block-Jacobi hot path.
+ *
+ * Method: H. Anzt, J. Dongarra, G. Flegar, E. S. Quintana-Orti, "Variable-Size
+ * Batched LU for Small Matrices and its Integration into Block-Jacobi
+ * Preconditioning", ICPP 2017.  "P:n" cites line n of the paper text
+ * with the section / figure it falls in; "R#" cites
+ * a reading of a silent or garbled passage, listed in DESIGN.md section 3.
+ *
+ * Conventions shared by every call
+ *  - Pointers are DEVICE pointers (cudaMalloc / torch CUDA tensors) unless the
+ *    parameter name ends in _h (HOST pointer).
+ *  - Calls are stream-ordered and asynchronous on `stream` (a cudaStream_t,
+ *    NULL = legacy default stream); none synchronises the host except those
+ *    documented as synchronous (bj_gesv_host).  The caller keeps every buffer
+ *    alive until the stream work completes.
+ *  - The library never allocates or frees caller data.  Library-owned memory
+ *    is limited to plan metadata (bj_plan, bj_handle, bj_workspace) and
+ *    stream-ordered scratch (cudaMallocAsync / cudaFreeAsync).
+ *  - Dense blocks are column-major, D(i,j) = values[val_off[b] + i + j*m]
+ *    (P:520-524), packed back to back; block b starts at element val_off[b],
+ *    which must be a multiple of 16/sizeof(element) (16-byte aligned, R18).
+ *    Vectors (pivots, right-hand sides, solutions) of block b start at element
+ *    vec_off[b].  bj_layout produces exactly this layout.
+ *  - Block orders m must lie in 0..32 (R10).  A block of
+ *    any other order gets info[b] = -1 and is not touched; there is no CPU or
+ *    other fallback path.
+ *  - Return value: BJ_OK, or a host-detectable error (bad arguments, launch
+ *    failure).  Data errors found on the device are reported per block in
+ *    info[] without a host synchronisation.
+ *  - Calls are reentrant; one bj_plan / bj_handle / bj_workspace must not be
+ *    used from two host threads at once.
+ */
+#ifndef BJ_H
+#define BJ_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *bj_stream_t;      /* == cudaStream_t */
+
+typedef enum { BJ_F32 = 0, BJ_F64 = 1 } bj_dtype;
+
+typedef enum {
+    BJ_OK = 0,
+    BJ_ERR_ARG = -1,         /* null pointer, negative count, bad dtype, ...   */
+    BJ_ERR_BLOCK_SIZE = -2,  /* reserved: sizes are checked per block (info=-1) */
+    BJ_ERR_ALIGN = -3,       /* a base pointer is not 16-byte aligned          */
+    BJ_ERR_CUDA = -4,        /* a CUDA runtime call or launch failed           */
+    BJ_ERR_NOMEM = -5,       /* library scratch allocation failed              */
+    BJ_ERR_STATE = -6        /* handle used before bj_setup, ...               */
+} bj_status;
+
+/* Sparse matrix in CSR (CSR [3]; Fig. 3).  Rows are
+ * local (0..nrows-1); col_idx holds GLOBAL column ids; local column =
+ * col_idx - col_offset (0 for a whole matrix; the first global row of a row
+ * slab when rows are sharded over GPUs).  Columns inside a row may be
+ * unsorted; (row, col) pairs must be unique (R14). */
+typedef struct {
+    int64_t nrows;
+    int64_t nnz;
+    int64_t col_offset;
+    const int64_t *row_ptr;      /* [nrows+1]                                 */
+    const int32_t *col_idx;      /* [nnz]                                     */
+    const void    *values;       /* [nnz] of dtype                            */
+    bj_dtype dtype;
+} bj_csr;
+
+/* A packed batch of dense blocks (layout above).  `values` is read and/or
+ * written depending on the call; the other arrays are inputs unless a call
+ * says it fills them. */
+typedef struct {
+    int64_t nblocks;
+    int32_t *sizes;              /* [nblocks]   block orders m_b              */
+    int64_t *vec_off;            /* [nblocks+1] exclusive prefix of m_b        */
+    int64_t *val_off;            /* [nblocks+1] element offset of block b      */
+    void    *values;             /* [val_off[nblocks]] elements of dtype       */
+    bj_dtype dtype;
+} bj_batch;
+
+/* Opaque objects (library-owned device metadata). */
+typedef struct bj_plan bj_plan;
+typedef struct bj_handle bj_handle;
+typedef struct bj_workspace bj_workspace;
+
+const char *bj_status_string(bj_status st);
+const char *bj_version(void);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a1 -- batch layout.  n = sum m_b.
+ *   vec_off[b] = sum_{c<b} m_c;  val_off[b] = sum_{c<b} roundup(m_c^2, 16/s)
+ * with s = sizeof(dtype); both int64[nblocks+1] (last entry = totals).
+ * Negative sizes count as 0.  Device scans; asynchronous.
+ * ------------------------------------------------------------------------- */
+bj_status bj_layout(int64_t nblocks, const int32_t *sizes, bj_dtype dtype,
+                    int64_t *vec_off, int64_t *val_off, bj_stream_t stream);
+
+/* Same layout from block boundaries (R15): sizes[b] = block_ptr[b+1] -
+ * block_ptr[b] is written to `sizes`, vec_off[b] = block_ptr[b] - block_ptr[0]. */
+bj_status bj_layout_from_block_ptr(int64_t nblocks, const int32_t *block_ptr, bj_dtype dtype,
+                                   int32_t *sizes, int64_t *vec_off, int64_t *val_off,
+                                   bj_stream_t stream);
+
+/* Size-bucket plan: block ids grouped by order m (stable counting sort on the
+ * device) and per-bucket task tables for the size-specialised kernels.  Reused
+ * by every call that receives it while `sizes` is unchanged.  Asynchronous;
+ * `sizes` must stay valid until the plan is destroyed only if the caller
+ * wants to reuse it (the plan copies what it needs). */
+bj_status bj_plan_create(bj_plan **plan, int64_t nblocks, const int32_t *sizes,
+                         bj_stream_t stream);
+bj_status bj_plan_destroy(bj_plan *plan);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a2 -- diagonal-block extraction, section III.C,
+ * block-Jacobi splitting P:159-171.
+ * For block b with rows bs = block_ptr[b] .. be = block_ptr[b+1]-1 (local
+ * rows; block columns are bs..be-1 in local column numbering):
+ *   D_b(r, c) = A(bs+r, bs+c) for every stored entry of row bs+r whose local
+ *   column lies in [bs, be); every other element of D_b is +0.0.
+ * Values are copied bit for bit.  `out` must carry the layout of
+ * bj_layout_from_block_ptr(block_ptr) (sizes/vec_off/val_off filled by the
+ * caller or by that call); out->values receives the blocks (pad elements
+ * between blocks are written as +0.0).  Rows with more than a few thousand
+ * stored entries are handled cooperatively (load balance for skewed rows).
+ * ------------------------------------------------------------------------- */
+bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out,
+                     bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a3 -- GETRF with implicit (swap-free) partial pivoting,
+ * Fig. 1 bottom, section III.A.
+ * Per block, for k = 0..m-1: pivot = the unpivoted row with the largest |a_ik|
+ * (bits of |a| compared as unsigned, the lowest original row wins ties, R1/R2);
+ * tag it; SCAL a_ik /= a_pk (IEEE division, R3) and GER a_ij = fma(-a_ik,
+ * a_pj, a_ij) on the unpivoted rows (R5); rows are finally stored in pivot
+ * order (combined row swap), giving P*D = L*U with unit-lower L
+ * (diagonal not stored) and upper U in place of D.
+ *   pivots[vec_off[b] + k] = original (0-based) row chosen at step k (R7).
+ *   info[b] = 0, or k+1 for the first step whose candidates are all +-0 (that
+ *   step's SCAL/GER are skipped, R4), or -1 if m_b is outside 0..32.
+ * `plan` may be NULL (a transient plan is built on `stream`).
+ * ------------------------------------------------------------------------- */
+bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info,
+                            const bj_plan *plan, bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a4 -- GETRS: x_b = D_b^{-1} b_b from the factors
+ * steps 2-4, Fig. 2 bottom and the mirrored upper solve (R8):
+ *   y = P b; eager unit-lower solve; eager upper solve with
+ *   y_k /= U(k,k) (IEEE division); x = y.
+ * b and x are packed at lu->vec_off; x may alias b exactly (not partially).
+ * Blocks whose order is outside 0..32 are skipped (x untouched).
+ * ------------------------------------------------------------------------- */
+bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const void *b, void *x,
+                            const bj_plan *plan, bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a5 -- block-Jacobi preconditioner, section II.A:
+ * setup = extract + factor every diagonal block,
+ * apply   y = D^{-1} x, one GETRS per block over the segments
+ *         x[block_ptr[b] .. block_ptr[b+1]) ("once per step").
+ * bj_setup fills factors->sizes/vec_off/val_off (caller buffers of nblocks /
+ * nblocks+1 / nblocks+1 entries; factors->values must hold
+ * val_off[nblocks] elements -- size it with bj_layout_from_block_ptr first),
+ * extracts into factors->values, factors in place, and keeps references to
+ * factors, pivots, block_ptr and a size plan in the handle.  x and y have
+ * A->nrows entries of the factor dtype (local rows); y may alias x.
+ * ------------------------------------------------------------------------- */
+bj_status bj_create(bj_handle **handle);
+bj_status bj_setup(bj_handle *handle, const bj_csr *A, const int32_t *block_ptr,
+                   bj_batch *factors, int32_t *pivots, int32_t *info, bj_stream_t stream);
+bj_status bj_apply(bj_handle *handle, const void *x, void *y, bj_stream_t stream);
+bj_status bj_destroy(bj_handle *handle);
+
+/* ---------------------------------------------------------------------------
+ * Hot-path row a6 -- contiguous cost-balanced batch partitioner (multi-GPU;
+ * not in the paper, which is single-GPU P:648).  HOST function.
+ *   cost_b = m_b^2, P(i) = sum_{b<i} cost_b (int64),
+ *   bounds[0] = 0, bounds[G] = nblocks,
+ *   bounds[r] = min{ i : G*P(i) >= r*P(nblocks) } for 0 < r < G   (R19).
+ * Rank r owns blocks [bounds[r], bounds[r+1]).
+ * ------------------------------------------------------------------------- */
+bj_status bj_partition(int64_t nblocks, const int32_t *sizes_h, int G, int64_t *bounds_h);
+
+/* ---------------------------------------------------------------------------
+ * End-to-end call with HOST buffers (synchronous): copies sizes_h (nblocks),
+ * blocks_h (nvalues elements, packed per bj_layout) and b_h (nvec elements)
+ * to the device, runs layout + plan + GETRF + GETRS, and copies x_h (nvec),
+ * pivots_h (nvec, may be NULL) and info_h (nblocks, may be NULL) back.
+ * Device buffers live in `ws` and grow on demand.  Host buffers should be
+ * pinned (cudaHostAlloc / torch pin_memory) for full PCIe bandwidth.
+ * ------------------------------------------------------------------------- */
+bj_status bj_workspace_create(bj_workspace **ws);
+bj_status bj_workspace_destroy(bj_workspace *ws);
+bj_status bj_gesv_host(bj_workspace *ws, int64_t nblocks, const int32_t *sizes_h,
+                       int64_t nvalues, const void *blocks_h, int64_t nvec, const void *b_h,
+                       void *x_h, int32_t *pivots_h, int32_t *info_h, bj_dtype dtype,
+                       bj_stream_t stream);
+
+/* Kernel launches issued by this library on the calling thread since the
+ * last reset (for the bench's gpu_launches count). */
+int64_t bj_launch_count(void);
+void bj_launch_count_reset(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BJ_H */

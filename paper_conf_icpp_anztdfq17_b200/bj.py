@@ -1,0 +1,338 @@
+"""Thin Python binding of the C ABI in include/bj.h (ctypes).
+
+Argument marshalling only: every step of the hot path runs in libbj.so's
+CUDA kernels.  PyTorch supplies device memory (``tensor.data_ptr()``) and the
+stream (``torch.cuda.current_stream().cuda_stream``).  There is no CPU
+fallback: if libbj.so is missing or a call fails, an exception is raised.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbj.so")
+
+BJ_F32, BJ_F64 = 0, 1
+_STATUS = {0: "BJ_OK", -1: "BJ_ERR_ARG", -2: "BJ_ERR_BLOCK_SIZE", -3: "BJ_ERR_ALIGN", -4: "BJ_ERR_CUDA",
+           -5: "BJ_ERR_NOMEM", -6: "BJ_ERR_STATE"}
+
+# every symbol include/bj.h and include/bj_synth.h declare
+EXPORTS = (
+    "bj_status_string", "bj_version", "bj_layout", "bj_layout_from_block_ptr", "bj_plan_create",
+    "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_create", "bj_setup",
+    "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
+    "bj_launch_count", "bj_launch_count_reset",
+    "bj_synth_sizes", "bj_synth_blocks", "bj_synth_rhs", "bj_synth_fem_row_ptr", "bj_synth_fem_fill",
+)
+
+
+class BJError(RuntimeError):
+    pass
+
+
+class CSR(ctypes.Structure):
+    _fields_ = [("nrows", ctypes.c_int64), ("nnz", ctypes.c_int64), ("col_offset", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("values", ctypes.c_void_p),
+                ("dtype", ctypes.c_int)]
+
+
+class BatchC(ctypes.Structure):
+    _fields_ = [("nblocks", ctypes.c_int64), ("sizes", ctypes.c_void_p), ("vec_off", ctypes.c_void_p),
+                ("val_off", ctypes.c_void_p), ("values", ctypes.c_void_p), ("dtype", ctypes.c_int)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libbj.so (fails loudly if it has not been built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise BJError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                          "(python -m paper_conf_icpp_anztdfq17_b200.build); there is no fallback path")
+        L = ctypes.CDLL(LIB_PATH)
+        P, I64, I32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+        sig = {
+            "bj_status_string": ([I32], ctypes.c_char_p),
+            "bj_version": ([], ctypes.c_char_p),
+            "bj_layout": ([I64, P, I32, P, P, P], I32),
+            "bj_layout_from_block_ptr": ([I64, P, I32, P, P, P, P], I32),
+            "bj_plan_create": ([P, I64, P, P], I32),
+            "bj_plan_destroy": ([P], I32),
+            "bj_extract": ([P, P, P, P], I32),
+            "bj_getrf_vbatched": ([P, P, P, P, P], I32),
+            "bj_getrs_vbatched": ([P, P, P, P, P, P], I32),
+            "bj_create": ([P], I32),
+            "bj_setup": ([P, P, P, P, P, P, P], I32),
+            "bj_apply": ([P, P, P, P], I32),
+            "bj_destroy": ([P], I32),
+            "bj_partition": ([I64, P, I32, P], I32),
+            "bj_workspace_create": ([P], I32),
+            "bj_workspace_destroy": ([P], I32),
+            "bj_gesv_host": ([P, I64, P, I64, P, I64, P, P, P, P, I32, P], I32),
+            "bj_launch_count": ([], I64),
+            "bj_launch_count_reset": ([], None),
+            "bj_synth_sizes": ([I64, I64, I32, I32, ctypes.c_uint64, P, P], I32),
+            "bj_synth_blocks": ([P, I64, I32, P], I32),
+            "bj_synth_rhs": ([P, I64, P, P], I32),
+            "bj_synth_fem_row_ptr": ([I32, I32, I32, I32, I64, I64, P, P], I32),
+            "bj_synth_fem_fill": ([I32, I32, I32, I32, I64, I64, P, P, P, I32, P], I32),
+        }
+        for name, (args, res) in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(st: int, what: str):
+    if st != 0:
+        raise BJError(f"{what}: {_STATUS.get(st, st)}")
+
+
+def _stream(stream=None) -> ctypes.c_void_p:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _p(t: torch.Tensor | None):
+    return ctypes.c_void_p(t.data_ptr()) if t is not None else None
+
+
+def dtype_code(dt: torch.dtype) -> int:
+    if dt == torch.float64:
+        return BJ_F64
+    if dt == torch.float32:
+        return BJ_F32
+    raise TypeError(f"unsupported dtype {dt}")
+
+
+def version() -> str:
+    return lib().bj_version().decode()
+
+
+def launch_count() -> int:
+    return int(lib().bj_launch_count())
+
+
+def launch_count_reset():
+    lib().bj_launch_count_reset()
+
+
+# --------------------------------------------------------------------------
+# batches
+# --------------------------------------------------------------------------
+@dataclass
+class Batch:
+    """Packed dense blocks (layout of include/bj.h).  All tensors on one CUDA
+    device: sizes int32[nb], vec_off/val_off int64[nb+1], values fp32/fp64."""
+    sizes: torch.Tensor
+    vec_off: torch.Tensor
+    val_off: torch.Tensor
+    values: torch.Tensor
+
+    @property
+    def nblocks(self) -> int:
+        return int(self.sizes.numel())
+
+    def c(self) -> BatchC:
+        return BatchC(self.nblocks, self.sizes.data_ptr(), self.vec_off.data_ptr(), self.val_off.data_ptr(),
+                      self.values.data_ptr(), dtype_code(self.values.dtype))
+
+
+def layout(sizes: torch.Tensor, dtype: torch.dtype, stream=None):
+    """Hot-path row a1: (vec_off, val_off) int64[nb+1] on sizes' device."""
+    nb = sizes.numel()
+    vec = torch.empty(nb + 1, dtype=torch.int64, device=sizes.device)
+    val = torch.empty(nb + 1, dtype=torch.int64, device=sizes.device)
+    _check(lib().bj_layout(nb, _p(sizes), dtype_code(dtype), _p(vec), _p(val), _stream(stream)), "bj_layout")
+    return vec, val
+
+
+def layout_from_block_ptr(block_ptr: torch.Tensor, dtype: torch.dtype, stream=None):
+    nb = block_ptr.numel() - 1
+    sizes = torch.empty(max(nb, 0), dtype=torch.int32, device=block_ptr.device)
+    vec = torch.empty(nb + 1, dtype=torch.int64, device=block_ptr.device)
+    val = torch.empty(nb + 1, dtype=torch.int64, device=block_ptr.device)
+    _check(lib().bj_layout_from_block_ptr(nb, _p(block_ptr), dtype_code(dtype), _p(sizes), _p(vec), _p(val),
+                                          _stream(stream)), "bj_layout_from_block_ptr")
+    return sizes, vec, val
+
+
+def new_batch(sizes: torch.Tensor, dtype: torch.dtype, stream=None) -> Batch:
+    """Allocate a batch for `sizes` (values uninitialised).  Syncs once to size
+    the value buffer."""
+    vec, val = layout(sizes, dtype, stream)
+    total = int(val[-1].item()) if sizes.numel() else 0
+    values = torch.empty(max(total, 1), dtype=dtype, device=sizes.device)
+    return Batch(sizes, vec, val, values)
+
+
+class Plan:
+    """Size-bucket plan (bj_plan_create); reuse across calls on the same sizes."""
+
+    def __init__(self, sizes: torch.Tensor, stream=None):
+        self._h = ctypes.c_void_p()
+        self.nblocks = sizes.numel()
+        _check(lib().bj_plan_create(ctypes.byref(self._h), self.nblocks, _p(sizes), _stream(stream)),
+               "bj_plan_create")
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if self._h:
+            lib().bj_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def getrf(batch: Batch, pivots: torch.Tensor, info: torch.Tensor, plan: Plan | None = None, stream=None):
+    """Hot-path row a3: in-place LU with implicit pivoting."""
+    b = batch.c()
+    _check(lib().bj_getrf_vbatched(ctypes.byref(b), _p(pivots), _p(info), plan.handle if plan else None,
+                                   _stream(stream)), "bj_getrf_vbatched")
+
+
+def getrs(batch: Batch, pivots: torch.Tensor, rhs: torch.Tensor, x: torch.Tensor, plan: Plan | None = None,
+          stream=None):
+    """Hot-path row a4: x = D^{-1} rhs per block (x may be rhs)."""
+    b = batch.c()
+    _check(lib().bj_getrs_vbatched(ctypes.byref(b), _p(pivots), _p(rhs), _p(x), plan.handle if plan else None,
+                                   _stream(stream)), "bj_getrs_vbatched")
+
+
+@dataclass
+class Csr:
+    row_ptr: torch.Tensor     # int64[nrows+1]
+    col_idx: torch.Tensor     # int32[nnz]
+    values: torch.Tensor      # fp32/fp64[nnz]
+    col_offset: int = 0
+
+    def c(self) -> CSR:
+        return CSR(self.row_ptr.numel() - 1, self.col_idx.numel(), int(self.col_offset), self.row_ptr.data_ptr(),
+                   self.col_idx.data_ptr(), self.values.data_ptr(), dtype_code(self.values.dtype))
+
+
+def extract(A: Csr, block_ptr: torch.Tensor, out: Batch, stream=None):
+    """Hot-path row a2: dense diagonal blocks of A into `out` (layout of
+    layout_from_block_ptr(block_ptr))."""
+    a = A.c()
+    o = out.c()
+    _check(lib().bj_extract(ctypes.byref(a), _p(block_ptr), ctypes.byref(o), _stream(stream)), "bj_extract")
+
+
+class Handle:
+    """Hot-path row a5: block-Jacobi preconditioner (setup = extract + getrf,
+    apply = getrs)."""
+
+    def __init__(self):
+        self._h = ctypes.c_void_p()
+        _check(lib().bj_create(ctypes.byref(self._h)), "bj_create")
+        self._keep = None
+
+    def setup(self, A: Csr, block_ptr: torch.Tensor, factors: Batch, pivots: torch.Tensor, info: torch.Tensor,
+              stream=None):
+        a = A.c()
+        f = factors.c()
+        _check(lib().bj_setup(self._h, ctypes.byref(a), _p(block_ptr), ctypes.byref(f), _p(pivots), _p(info),
+                              _stream(stream)), "bj_setup")
+        self._keep = (A, block_ptr, factors, pivots, info)
+
+    def apply(self, x: torch.Tensor, y: torch.Tensor, stream=None):
+        _check(lib().bj_apply(self._h, _p(x), _p(y), _stream(stream)), "bj_apply")
+
+    def close(self):
+        if self._h:
+            lib().bj_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def partition(sizes: np.ndarray, G: int) -> np.ndarray:
+    """Hot-path row a6 (host): contiguous cost-balanced shard boundaries."""
+    s = np.ascontiguousarray(sizes, dtype=np.int32)
+    out = np.zeros(G + 1, dtype=np.int64)
+    _check(lib().bj_partition(s.shape[0], s.ctypes.data_as(ctypes.c_void_p), int(G),
+                              out.ctypes.data_as(ctypes.c_void_p)), "bj_partition")
+    return out
+
+
+class Workspace:
+    """Device workspace of bj_gesv_host (end-to-end call with host buffers)."""
+
+    def __init__(self):
+        self._h = ctypes.c_void_p()
+        _check(lib().bj_workspace_create(ctypes.byref(self._h)), "bj_workspace_create")
+
+    def gesv_host(self, sizes_h: torch.Tensor, blocks_h: torch.Tensor, b_h: torch.Tensor, x_h: torch.Tensor,
+                  pivots_h: torch.Tensor | None = None, info_h: torch.Tensor | None = None, stream=None):
+        _check(lib().bj_gesv_host(self._h, sizes_h.numel(), _p(sizes_h), blocks_h.numel(), _p(blocks_h),
+                                  b_h.numel(), _p(b_h), _p(x_h), _p(pivots_h), _p(info_h),
+                                  dtype_code(blocks_h.dtype), _stream(stream)), "bj_gesv_host")
+
+    def close(self):
+        if self._h:
+            lib().bj_workspace_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# --------------------------------------------------------------------------
+# device-side synthetic inputs (bj_synth.h)
+# --------------------------------------------------------------------------
+def synth_sizes(nb: int, lo: int, hi: int, first: int = 0, seed: int = 1, device="cuda", stream=None):
+    s = torch.empty(max(nb, 1), dtype=torch.int32, device=device)[:nb]
+    _check(lib().bj_synth_sizes(nb, first, lo, hi, seed, _p(s), _stream(stream)), "bj_synth_sizes")
+    return s
+
+
+def synth_blocks(batch: Batch, first: int = 0, kind: int = 0, stream=None):
+    b = batch.c()
+    _check(lib().bj_synth_blocks(ctypes.byref(b), first, kind, _stream(stream)), "bj_synth_blocks")
+
+
+def synth_rhs(batch: Batch, first: int = 0, stream=None) -> torch.Tensor:
+    n = int(batch.vec_off[-1].item()) if batch.nblocks else 0
+    out = torch.empty(max(n, 1), dtype=batch.values.dtype, device=batch.values.device)
+    b = batch.c()
+    _check(lib().bj_synth_rhs(ctypes.byref(b), first, _p(out), _stream(stream)), "bj_synth_rhs")
+    return out
+
+
+def synth_fem(nx: int, ny: int, nz: int, r0: int, r1: int, dtype=torch.float64, skew: bool = True,
+              device="cuda", stream=None) -> Csr:
+    """FEM-like CSR rows [r0, r1) (local rows, global columns; col_offset=r0)."""
+    n = r1 - r0
+    rp = torch.empty(n + 1, dtype=torch.int64, device=device)
+    _check(lib().bj_synth_fem_row_ptr(nx, ny, nz, int(skew), r0, r1, _p(rp), _stream(stream)),
+           "bj_synth_fem_row_ptr")
+    nnz = int(rp[-1].item())
+    ci = torch.empty(max(nnz, 1), dtype=torch.int32, device=device)
+    va = torch.empty(max(nnz, 1), dtype=dtype, device=device)
+    _check(lib().bj_synth_fem_fill(nx, ny, nz, int(skew), r0, r1, _p(rp), _p(ci), _p(va), dtype_code(dtype),
+                                   _stream(stream)), "bj_synth_fem_fill")
+    return Csr(rp, ci[:nnz], va[:nnz], r0)

@@ -1,0 +1,330 @@
+// api.cu -- the C ABI (include/bj.h): argument checking, plans, handles,
+// workspaces and dispatch to the kernel translation units.  No arithmetic of
+// the method lives here; there is no CPU or library fallback.
+#include <new>
+#include <string.h>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace bj {
+
+static thread_local int64_t g_launches = 0;
+void count_launch(int n) { g_launches += n; }
+
+int sm_count() {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static int cached[64] = {0};
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (cached[dev] == 0) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        cached[dev] = n > 0 ? n : 1;
+    }
+    return cached[dev];
+}
+
+static int elem_size(bj_dtype d) { return d == BJ_F64 ? 8 : d == BJ_F32 ? 4 : 0; }
+static bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+
+static bj_status check_batch(const bj_batch *b, bool need_values) {
+    if (!b || b->nblocks < 0 || elem_size(b->dtype) == 0) return BJ_ERR_ARG;
+    if (b->nblocks > 0 && (!b->sizes || !b->vec_off || !b->val_off)) return BJ_ERR_ARG;
+    if (need_values && b->nblocks > 0 && !b->values) return BJ_ERR_ARG;
+    if (b->values && !aligned16(b->values)) return BJ_ERR_ALIGN;
+    if (b->nblocks >= (int64_t)1 << 31) return BJ_ERR_ARG;   // block ids are int32
+    return BJ_OK;
+}
+
+}  // namespace bj
+
+using namespace bj;
+
+struct bj_plan {
+    int64_t nblocks = 0;
+    int32_t *order = nullptr;
+    int64_t *bin_start = nullptr;
+    PlanView view() const { return PlanView{nblocks, order, bin_start}; }
+};
+
+struct bj_handle {
+    bool ready = false;
+    bj_batch factors{};
+    int32_t *pivots = nullptr;
+    bj_plan plan;
+    int64_t nrows = 0;
+};
+
+struct bj_workspace {
+    char *dev = nullptr;
+    size_t cap = 0;
+};
+
+static bj_status plan_alloc_build(bj_plan *p, int64_t nb, const int32_t *sizes, cudaStream_t s) {
+    p->nblocks = nb;
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&p->order, sizeof(int32_t) * (size_t)(nb > 0 ? nb : 1), s));
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&p->bin_start, sizeof(int64_t) * (kBins + 1), s));
+    return build_plan(nb, sizes, p->order, p->bin_start, s);
+}
+
+static void plan_free_async(bj_plan *p, cudaStream_t s) {
+    if (p->order) cudaFreeAsync(p->order, s);
+    if (p->bin_start) cudaFreeAsync(p->bin_start, s);
+    p->order = nullptr;
+    p->bin_start = nullptr;
+}
+
+extern "C" {
+
+const char *bj_status_string(bj_status st) {
+    switch (st) {
+    case BJ_OK: return "BJ_OK";
+    case BJ_ERR_ARG: return "BJ_ERR_ARG: invalid argument";
+    case BJ_ERR_BLOCK_SIZE: return "BJ_ERR_BLOCK_SIZE: block order outside 0..32";
+    case BJ_ERR_ALIGN: return "BJ_ERR_ALIGN: pointer not 16-byte aligned";
+    case BJ_ERR_CUDA: return "BJ_ERR_CUDA: CUDA runtime error";
+    case BJ_ERR_NOMEM: return "BJ_ERR_NOMEM: allocation failed";
+    case BJ_ERR_STATE: return "BJ_ERR_STATE: object not ready";
+    }
+    return "unknown bj_status";
+}
+
+const char *bj_version(void) { return "bj-b200 0.1 (sm_100a)"; }
+
+int64_t bj_launch_count(void) { return g_launches; }
+void bj_launch_count_reset(void) { g_launches = 0; }
+
+bj_status bj_layout(int64_t nblocks, const int32_t *sizes, bj_dtype dtype, int64_t *vec_off, int64_t *val_off,
+                    bj_stream_t stream) {
+    const int es = elem_size(dtype);
+    if (nblocks < 0 || es == 0 || !vec_off || !val_off || (nblocks > 0 && !sizes)) return BJ_ERR_ARG;
+    return layout_sizes(nblocks, sizes, es, vec_off, val_off, (cudaStream_t)stream);
+}
+
+bj_status bj_layout_from_block_ptr(int64_t nblocks, const int32_t *block_ptr, bj_dtype dtype, int32_t *sizes,
+                                   int64_t *vec_off, int64_t *val_off, bj_stream_t stream) {
+    const int es = elem_size(dtype);
+    if (nblocks < 0 || es == 0 || !block_ptr || !vec_off || !val_off || (nblocks > 0 && !sizes)) return BJ_ERR_ARG;
+    return layout_block_ptr(nblocks, block_ptr, es, sizes, vec_off, val_off, (cudaStream_t)stream);
+}
+
+bj_status bj_plan_create(bj_plan **plan, int64_t nblocks, const int32_t *sizes, bj_stream_t stream) {
+    if (!plan || nblocks < 0 || (nblocks > 0 && !sizes) || nblocks >= (int64_t)1 << 31) return BJ_ERR_ARG;
+    bj_plan *p = new (std::nothrow) bj_plan();
+    if (!p) return BJ_ERR_NOMEM;
+    bj_status st = plan_alloc_build(p, nblocks, sizes, (cudaStream_t)stream);
+    if (st != BJ_OK) {
+        plan_free_async(p, (cudaStream_t)stream);
+        delete p;
+        return st;
+    }
+    *plan = p;
+    return BJ_OK;
+}
+
+bj_status bj_plan_destroy(bj_plan *plan) {
+    if (!plan) return BJ_ERR_ARG;
+    if (plan->order) cudaFree(plan->order);
+    if (plan->bin_start) cudaFree(plan->bin_start);
+    delete plan;
+    return BJ_OK;
+}
+
+bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out, bj_stream_t stream) {
+    if (!A || !block_ptr) return BJ_ERR_ARG;
+    bj_status st = check_batch(out, true);
+    if (st != BJ_OK) return st;
+    if (A->dtype != out->dtype || A->nrows < 0 || A->nnz < 0 || !A->row_ptr) return BJ_ERR_ARG;
+    if (A->nnz > 0 && (!A->col_idx || !A->values)) return BJ_ERR_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (out->dtype == BJ_F64)
+        return extract_run<double>(*A, block_ptr, out->nblocks, out->val_off, (double *)out->values, s);
+    return extract_run<float>(*A, block_ptr, out->nblocks, out->val_off, (float *)out->values, s);
+}
+
+bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const bj_plan *plan,
+                            bj_stream_t stream) {
+    bj_status st = check_batch(blocks, true);
+    if (st != BJ_OK) return st;
+    if (blocks->nblocks > 0 && (!pivots || !info)) return BJ_ERR_ARG;
+    if (plan && plan->nblocks != blocks->nblocks) return BJ_ERR_ARG;
+    if (blocks->nblocks == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    bj_plan tmp;
+    const bj_plan *p = plan;
+    if (!p) {
+        if ((st = plan_alloc_build(&tmp, blocks->nblocks, blocks->sizes, s)) != BJ_OK) {
+            plan_free_async(&tmp, s);
+            return st;
+        }
+        p = &tmp;
+    }
+    if (blocks->dtype == BJ_F64)
+        st = getrf_run<double>((double *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(), s);
+    else
+        st = getrf_run<float>((float *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(), s);
+    if (!plan) plan_free_async(&tmp, s);
+    return st;
+}
+
+bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const void *b, void *x, const bj_plan *plan,
+                            bj_stream_t stream) {
+    bj_status st = check_batch(lu, true);
+    if (st != BJ_OK) return st;
+    if (lu->nblocks > 0 && (!pivots || !b || !x)) return BJ_ERR_ARG;
+    if (plan && plan->nblocks != lu->nblocks) return BJ_ERR_ARG;
+    if (lu->nblocks == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    bj_plan tmp;
+    const bj_plan *p = plan;
+    if (!p) {
+        if ((st = plan_alloc_build(&tmp, lu->nblocks, lu->sizes, s)) != BJ_OK) {
+            plan_free_async(&tmp, s);
+            return st;
+        }
+        p = &tmp;
+    }
+    if (lu->dtype == BJ_F64)
+        st = getrs_run<double>((const double *)lu->values, lu->val_off, lu->vec_off, pivots, (const double *)b,
+                               (double *)x, p->view(), s);
+    else
+        st = getrs_run<float>((const float *)lu->values, lu->val_off, lu->vec_off, pivots, (const float *)b,
+                              (float *)x, p->view(), s);
+    if (!plan) plan_free_async(&tmp, s);
+    return st;
+}
+
+bj_status bj_create(bj_handle **handle) {
+    if (!handle) return BJ_ERR_ARG;
+    bj_handle *h = new (std::nothrow) bj_handle();
+    if (!h) return BJ_ERR_NOMEM;
+    *handle = h;
+    return BJ_OK;
+}
+
+bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *factors, int32_t *pivots,
+                   int32_t *info, bj_stream_t stream) {
+    if (!h || !A || !block_ptr || !factors) return BJ_ERR_ARG;
+    bj_status st = check_batch(factors, true);
+    if (st != BJ_OK) return st;
+    if (A->dtype != factors->dtype) return BJ_ERR_ARG;
+    if (factors->nblocks > 0 && (!pivots || !info)) return BJ_ERR_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t nb = factors->nblocks;
+    const int es = elem_size(factors->dtype);
+    h->ready = false;
+    if ((st = layout_block_ptr(nb, block_ptr, es, factors->sizes, factors->vec_off, factors->val_off, s)) != BJ_OK)
+        return st;
+    if ((st = bj_extract(A, block_ptr, factors, stream)) != BJ_OK) return st;
+    plan_free_async(&h->plan, s);
+    if ((st = plan_alloc_build(&h->plan, nb, factors->sizes, s)) != BJ_OK) return st;
+    if ((st = bj_getrf_vbatched(factors, pivots, info, &h->plan, stream)) != BJ_OK) return st;
+    h->factors = *factors;
+    h->pivots = pivots;
+    h->nrows = A->nrows;
+    h->ready = true;
+    return BJ_OK;
+}
+
+bj_status bj_apply(bj_handle *h, const void *x, void *y, bj_stream_t stream) {
+    if (!h || !x || !y) return BJ_ERR_ARG;
+    if (!h->ready) return BJ_ERR_STATE;
+    return bj_getrs_vbatched(&h->factors, h->pivots, x, y, &h->plan, stream);
+}
+
+bj_status bj_destroy(bj_handle *h) {
+    if (!h) return BJ_ERR_ARG;
+    if (h->plan.order) cudaFree(h->plan.order);
+    if (h->plan.bin_start) cudaFree(h->plan.bin_start);
+    delete h;
+    return BJ_OK;
+}
+
+bj_status bj_partition(int64_t nblocks, const int32_t *sizes_h, int G, int64_t *bounds_h) {
+    if (nblocks < 0 || G < 1 || !bounds_h || (nblocks > 0 && !sizes_h)) return BJ_ERR_ARG;
+    int64_t total = 0;
+    for (int64_t i = 0; i < nblocks; ++i) total += (int64_t)sizes_h[i] * sizes_h[i];
+    bounds_h[0] = 0;
+    bounds_h[G] = nblocks;
+    // single sweep: boundary r is the first i with G*P(i) >= r*total
+    int64_t P = 0, i = 0;
+    for (int r = 1; r < G; ++r) {
+        const __int128 target = (__int128)r * total;
+        while (i < nblocks && (__int128)G * P < target) {
+            P += (int64_t)sizes_h[i] * sizes_h[i];
+            ++i;
+        }
+        bounds_h[r] = i;
+    }
+    return BJ_OK;
+}
+
+bj_status bj_workspace_create(bj_workspace **ws) {
+    if (!ws) return BJ_ERR_ARG;
+    bj_workspace *w = new (std::nothrow) bj_workspace();
+    if (!w) return BJ_ERR_NOMEM;
+    *ws = w;
+    return BJ_OK;
+}
+
+bj_status bj_workspace_destroy(bj_workspace *ws) {
+    if (!ws) return BJ_ERR_ARG;
+    if (ws->dev) cudaFree(ws->dev);
+    delete ws;
+    return BJ_OK;
+}
+
+static size_t up256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int64_t nvalues, const void *blocks_h,
+                       int64_t nvec, const void *b_h, void *x_h, int32_t *pivots_h, int32_t *info_h, bj_dtype dtype,
+                       bj_stream_t stream) {
+    const int es = elem_size(dtype);
+    if (!ws || nb < 0 || nvalues < 0 || nvec < 0 || es == 0) return BJ_ERR_ARG;
+    if (nb > 0 && (!sizes_h || !blocks_h || !b_h || !x_h)) return BJ_ERR_ARG;
+    if (nb == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t o_sizes = 0;
+    const size_t o_vec = o_sizes + up256(sizeof(int32_t) * nb);
+    const size_t o_val = o_vec + up256(sizeof(int64_t) * (nb + 1));
+    const size_t o_A = o_val + up256(sizeof(int64_t) * (nb + 1));
+    const size_t o_b = o_A + up256((size_t)es * nvalues);
+    const size_t o_x = o_b + up256((size_t)es * nvec);
+    const size_t o_piv = o_x + up256((size_t)es * nvec);
+    const size_t o_info = o_piv + up256(sizeof(int32_t) * nvec);
+    const size_t o_order = o_info + up256(sizeof(int32_t) * nb);
+    const size_t o_bins = o_order + up256(sizeof(int32_t) * nb);
+    const size_t need = o_bins + up256(sizeof(int64_t) * (kBins + 1));
+    if (need > ws->cap) {
+        if (ws->dev) BJ_CUDA_TRY(cudaFree(ws->dev));
+        ws->dev = nullptr;
+        ws->cap = 0;
+        if (cudaMalloc((void **)&ws->dev, need) != cudaSuccess) return BJ_ERR_NOMEM;
+        ws->cap = need;
+    }
+    char *d = ws->dev;
+    int32_t *sizes = (int32_t *)(d + o_sizes);
+    int64_t *vec = (int64_t *)(d + o_vec), *val = (int64_t *)(d + o_val);
+    int32_t *piv = (int32_t *)(d + o_piv), *info = (int32_t *)(d + o_info);
+    BJ_CUDA_TRY(cudaMemcpyAsync(sizes, sizes_h, sizeof(int32_t) * nb, cudaMemcpyHostToDevice, s));
+    BJ_CUDA_TRY(cudaMemcpyAsync(d + o_A, blocks_h, (size_t)es * nvalues, cudaMemcpyHostToDevice, s));
+    BJ_CUDA_TRY(cudaMemcpyAsync(d + o_b, b_h, (size_t)es * nvec, cudaMemcpyHostToDevice, s));
+    bj_status st;
+    if ((st = layout_sizes(nb, sizes, es, vec, val, s)) != BJ_OK) return st;
+    bj_plan p;
+    p.nblocks = nb;
+    p.order = (int32_t *)(d + o_order);
+    p.bin_start = (int64_t *)(d + o_bins);
+    if ((st = build_plan(nb, sizes, p.order, p.bin_start, s)) != BJ_OK) return st;
+    bj_batch batch{nb, sizes, vec, val, d + o_A, dtype};
+    if ((st = bj_getrf_vbatched(&batch, piv, info, &p, stream)) != BJ_OK) return st;
+    if ((st = bj_getrs_vbatched(&batch, piv, d + o_b, d + o_x, &p, stream)) != BJ_OK) return st;
+    BJ_CUDA_TRY(cudaMemcpyAsync(x_h, d + o_x, (size_t)es * nvec, cudaMemcpyDeviceToHost, s));
+    if (pivots_h) BJ_CUDA_TRY(cudaMemcpyAsync(pivots_h, piv, sizeof(int32_t) * nvec, cudaMemcpyDeviceToHost, s));
+    if (info_h) BJ_CUDA_TRY(cudaMemcpyAsync(info_h, info, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost, s));
+    BJ_CUDA_TRY(cudaStreamSynchronize(s));
+    return BJ_OK;
+}
+
+}  // extern "C"

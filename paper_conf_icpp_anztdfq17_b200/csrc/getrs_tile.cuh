@@ -1,0 +1,45 @@
+// getrs_tile.cuh -- one warp-tile of GETRS (used by getrs.cu and by the
+// block-Jacobi apply, which is the same solve over global-vector segments).
+#pragma once
+
+#include "common.cuh"
+
+namespace bj {
+
+// LU: this tile's block (column-major, rows in pivot order), piv/b/x: this
+// block's vector segments.  Each lane of the tile handles one row.
+template <typename R, int M>
+__device__ __forceinline__ void getrs_tile(const R *__restrict__ LU, const int32_t *__restrict__ piv,
+                                           const R *b, R *x, bool tile_ok) {
+    constexpr int T = tile_width(M);
+    const int lane = threadIdx.x & 31;
+    const int r = lane % T;
+    const int tbase = lane - r;
+    const bool row_ok = tile_ok && (r < M);
+
+    R a[M];                                     // row r of L\U
+    static_for<0, M>([&](auto jc) {
+        constexpr int j = decltype(jc)::value;
+        a[j] = row_ok ? __ldg(LU + r + j * M) : R(0);
+    });
+    // b := P b: lane r receives b[perm[r]].
+    R y = row_ok ? b[__ldg(piv + r)] : R(0);
+
+    // L y = P b, eager (Fig. 2 bottom): y_i -= L(i,k) y_k for i > k.
+    static_for<0, M - 1>([&](auto kc) {
+        constexpr int k = decltype(kc)::value;
+        const R yk = __shfl_sync(kFull, y, tbase + k);
+        if (r > k) y = Num<R>::fma(-a[k], yk, y);
+    });
+    // U x = y, eager and mirrored (R8): y_k /= U(k,k); y_i -= U(i,k) y_k, i < k.
+    static_for<0, M>([&](auto kk) {
+        constexpr int k = M - 1 - decltype(kk)::value;
+        if (r == k) y = Num<R>::div(y, a[k]);
+        const R yk = __shfl_sync(kFull, y, tbase + k);
+        if (r < k) y = Num<R>::fma(-a[k], yk, y);
+    });
+    __syncwarp();                               // every lane has read b before x is written (x may alias b)
+    if (row_ok) x[r] = y;
+}
+
+}  // namespace bj

@@ -1,0 +1,172 @@
+// layout.cu -- hot-path row a1: batch layout (vec_off / val_off scans) and the
+// size-bucket plan (stable device counting sort of block ids by order m).
+//
+// The paper pads every block to 32 x 32; here blocks are packed
+// back to back (16-byte aligned starts) and grouped by exact order so the
+// size-specialised kernels never compute on padding.
+#include "scan.cuh"
+#include "internal.h"
+
+namespace bj {
+
+// ---------------------------------------------------------------- layout
+struct SizesLayoutF {
+    const int32_t *sizes;
+    int64_t *vec, *val;
+    int q;
+    __device__ I64x2 value(int64_t i) const {
+        long long m = max(sizes[i], 0);
+        long long sq = m * m;
+        return I64x2{m, (sq + q - 1) / q * q};
+    }
+    __device__ void store(int64_t i, I64x2 p) const { vec[i] = p.a; val[i] = p.b; }
+    bj_status store_empty(cudaStream_t s) const {
+        BJ_CUDA_TRY(cudaMemsetAsync(vec, 0, sizeof(int64_t), s));
+        BJ_CUDA_TRY(cudaMemsetAsync(val, 0, sizeof(int64_t), s));
+        return BJ_OK;
+    }
+};
+
+struct BlockPtrLayoutF {
+    const int32_t *bp;
+    int32_t *sizes;
+    int64_t *vec, *val;
+    int64_t n;
+    int q;
+    __device__ I64x2 value(int64_t i) const {
+        long long m = max(bp[i + 1] - bp[i], 0);
+        long long sq = m * m;
+        return I64x2{m, (sq + q - 1) / q * q};
+    }
+    __device__ void store(int64_t i, I64x2 p) const {
+        vec[i] = p.a;
+        val[i] = p.b;
+        if (i < n) sizes[i] = bp[i + 1] - bp[i];
+    }
+    bj_status store_empty(cudaStream_t s) const {
+        BJ_CUDA_TRY(cudaMemsetAsync(vec, 0, sizeof(int64_t), s));
+        BJ_CUDA_TRY(cudaMemsetAsync(val, 0, sizeof(int64_t), s));
+        return BJ_OK;
+    }
+};
+
+bj_status layout_sizes(int64_t nb, const int32_t *sizes, int elem, int64_t *vec, int64_t *val,
+                       cudaStream_t s) {
+    return run_scan(SizesLayoutF{sizes, vec, val, 16 / elem}, nb, s);
+}
+
+bj_status layout_block_ptr(int64_t nb, const int32_t *bp, int elem, int32_t *sizes, int64_t *vec,
+                           int64_t *val, cudaStream_t s) {
+    return run_scan(BlockPtrLayoutF{bp, sizes, vec, val, nb, 16 / elem}, nb, s);
+}
+
+// ---------------------------------------------------------------- plan
+// Tiles of kPlanTile consecutive blocks; per tile a histogram over the 34
+// bins, a global (bin, tile) prefix, then a stable scatter.
+constexpr int kPlanThreads = 256;
+constexpr int kPlanRounds = 8;
+constexpr int kPlanTile = kPlanThreads * kPlanRounds;
+
+__global__ void __launch_bounds__(kPlanThreads)
+k_plan_hist(const int32_t *__restrict__ sizes, int64_t n, int64_t *__restrict__ hist) {
+    __shared__ int cnt[kBins];
+    for (int i = threadIdx.x; i < kBins; i += blockDim.x) cnt[i] = 0;
+    __syncthreads();
+    const int64_t base = (int64_t)blockIdx.x * kPlanTile;
+    for (int j = 0; j < kPlanRounds; ++j) {
+        int64_t i = base + j * kPlanThreads + threadIdx.x;
+        if (i < n) atomicAdd(&cnt[size_bin(sizes[i])], 1);
+    }
+    __syncthreads();
+    for (int b = threadIdx.x; b < kBins; b += blockDim.x) hist[(int64_t)blockIdx.x * kBins + b] = cnt[b];
+}
+
+// Single CTA: hist[tile][bin] -> absolute start of (tile, bin) in `order`;
+// bin_start[bin] = start of bin (bin_start[kBins] = n).
+__global__ void __launch_bounds__(64) k_plan_offsets(int64_t *hist, int64_t ntiles, int64_t *bin_start) {
+    __shared__ int64_t tot[kBins];
+    const int b = threadIdx.x;
+    int64_t acc = 0;
+    if (b < kBins) {
+        for (int64_t t = 0; t < ntiles; ++t) {
+            int64_t c = hist[t * kBins + b];
+            hist[t * kBins + b] = acc;
+            acc += c;
+        }
+        tot[b] = acc;
+    }
+    __syncthreads();
+    if (b == 0) {
+        int64_t s = 0;
+        for (int i = 0; i < kBins; ++i) {
+            int64_t c = tot[i];
+            tot[i] = s;
+            bin_start[i] = s;
+            s += c;
+        }
+        bin_start[kBins] = s;
+    }
+    __syncthreads();
+    if (b < kBins) {
+        const int64_t s = tot[b];
+        for (int64_t t = 0; t < ntiles; ++t) hist[t * kBins + b] += s;
+    }
+}
+
+__global__ void __launch_bounds__(kPlanThreads)
+k_plan_scatter(const int32_t *__restrict__ sizes, int64_t n, const int64_t *__restrict__ tile_off,
+               int32_t *__restrict__ order) {
+    constexpr int NW = kPlanThreads / 32;
+    __shared__ int64_t run[kBins];               // offset of the next item of each bin
+    __shared__ int rtot[kBins];
+    __shared__ int wpre[NW][kBins];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int b = threadIdx.x; b < kBins; b += blockDim.x) run[b] = tile_off[(int64_t)blockIdx.x * kBins + b];
+    const int64_t base = (int64_t)blockIdx.x * kPlanTile;
+    const unsigned lt = (1u << lane) - 1u;
+    for (int j = 0; j < kPlanRounds; ++j) {
+        for (int b = threadIdx.x; b < NW * kBins; b += blockDim.x) (&wpre[0][0])[b] = 0;
+        __syncthreads();
+        const int64_t i = base + (int64_t)j * kPlanThreads + threadIdx.x;
+        const int bin = i < n ? size_bin(sizes[i]) : -1;
+        const unsigned peers = __match_any_sync(kFull, bin);
+        const int rank = __popc(peers & lt);     // stable rank inside the warp
+        if (bin >= 0 && rank == 0) wpre[w][bin] = __popc(peers);
+        __syncthreads();
+        if (threadIdx.x < kBins) {               // exclusive prefix over warps, per bin
+            const int b = threadIdx.x;
+            int acc = 0;
+            for (int ww = 0; ww < NW; ++ww) {
+                const int c = wpre[ww][b];
+                wpre[ww][b] = acc;
+                acc += c;
+            }
+            rtot[b] = acc;
+        }
+        __syncthreads();
+        if (bin >= 0) order[run[bin] + wpre[w][bin] + rank] = (int32_t)i;
+        __syncthreads();
+        if (threadIdx.x < kBins) run[threadIdx.x] += rtot[threadIdx.x];
+    }
+}
+
+bj_status build_plan(int64_t nb, const int32_t *sizes, int32_t *order, int64_t *bin_start,
+                     cudaStream_t s) {
+    if (nb == 0) {
+        BJ_CUDA_TRY(cudaMemsetAsync(bin_start, 0, sizeof(int64_t) * (kBins + 1), s));
+        return BJ_OK;
+    }
+    const int64_t ntiles = (nb + kPlanTile - 1) / kPlanTile;
+    int64_t *hist = nullptr;
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&hist, sizeof(int64_t) * kBins * ntiles, s));
+    k_plan_hist<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist);
+    BJ_LAUNCH_CHECK();
+    k_plan_offsets<<<1, 64, 0, s>>>(hist, ntiles, bin_start);
+    BJ_LAUNCH_CHECK();
+    k_plan_scatter<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist, order);
+    BJ_LAUNCH_CHECK();
+    BJ_CUDA_TRY(cudaFreeAsync(hist, s));
+    return BJ_OK;
+}
+
+}  // namespace bj

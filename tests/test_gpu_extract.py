@@ -1,0 +1,159 @@
+"""GPU parity of diagonal-block extraction (row a2) and of the block-Jacobi
+handle (row a5: setup = extract + getrf, apply = getrs) against the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import bj_synth as S
+import oracle
+from gpu_helpers import NP, bits
+from paper_conf_icpp_anztdfq17_b200 import bj
+
+pytestmark = pytest.mark.gpu
+
+
+def _extract_dev(rp, ci, va, bp, col_offset=0):
+    dtype = torch.float64 if va.dtype == np.float64 else torch.float32
+    A = bj.Csr(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), torch.from_numpy(va).cuda(), col_offset)
+    bpt = torch.from_numpy(bp).cuda()
+    sizes, vec, val = bj.layout_from_block_ptr(bpt, dtype)
+    total = int(val[-1].item())
+    out = bj.Batch(sizes, vec, val, torch.full((max(total, 1),), float("nan"), dtype=dtype, device="cuda"))
+    bj.extract(A, bpt, out)
+    torch.cuda.synchronize()
+    return out
+
+
+def _check(rp, ci, va, bp, col_offset=0):
+    out = _extract_dev(rp, ci, va, bp, col_offset)
+    ref, sizes, vec, val = oracle.extract(rp, ci, va, bp, col_offset)
+    assert np.array_equal(out.sizes.cpu().numpy(), sizes)
+    assert np.array_equal(out.val_off.cpu().numpy(), val)
+    got = out.values.cpu().numpy()
+    for b in range(len(sizes)):
+        m = int(sizes[b])
+        q = 16 // va.dtype.itemsize
+        a, e = int(val[b]), int(val[b]) + m * m
+        assert np.array_equal(bits(got[a:e]), bits(ref[a:e])), f"block {b}"
+        pad = got[e: int(val[b]) + (m * m + q - 1) // q * q]
+        assert np.all(bits(pad) == 0)                     # pad written as +0.0
+
+
+def _random_csr(rng, n, density, dtype):
+    rp = [0]
+    cols, vals = [], []
+    for r in range(n):
+        k = rng.binomial(n, density)
+        c = rng.choice(n, size=k, replace=False)
+        v = rng.uniform(-1, 1, size=k).astype(dtype)
+        if k:
+            v[rng.random(k) < 0.1] = -0.0
+        cols.append(c)
+        vals.append(v)
+        rp.append(rp[-1] + k)
+    return np.asarray(rp, np.int64), np.concatenate(cols).astype(np.int32), np.concatenate(vals).astype(dtype)
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_random_csr_unsorted(dtype):
+    rng = np.random.default_rng(41)
+    for _ in range(4):
+        n = int(rng.integers(100, 600))
+        rp, ci, va = _random_csr(rng, n, 0.08, dtype)
+        edges = [0]
+        while edges[-1] < n:
+            edges.append(min(n, edges[-1] + int(rng.integers(1, 33))))
+        _check(rp, ci, va, np.asarray(edges, np.int32))
+
+
+def test_heavy_rows_take_the_cta_path():
+    """Rows with far more than kHeavy entries (skewed nnz)."""
+    rng = np.random.default_rng(42)
+    n = 50000
+    rows = []
+    for r in range(n):
+        if r in (5, 17, 40000):
+            c = rng.choice(n, size=30000, replace=False)    # hub rows
+        else:
+            c = np.unique(np.clip(r + rng.integers(-20, 21, size=9), 0, n - 1))
+        rows.append(c)
+    rp = np.concatenate([[0], np.cumsum([len(c) for c in rows])]).astype(np.int64)
+    ci = np.concatenate(rows).astype(np.int32)
+    va = rng.uniform(-1, 1, size=len(ci))
+    _check(rp, ci, va, S.uniform_block_ptr(n, 24))
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_fem_small_grid_device_generator_and_extract(dtype):
+    g = S.FemGrid(13, 11, 9)
+    A = bj.synth_fem(13, 11, 9, 0, g.n, dtype=dtype)
+    rp, ci, va = g.csr(dtype=NP[dtype])
+    assert np.array_equal(A.row_ptr.cpu().numpy(), rp)
+    assert np.array_equal(A.col_idx.cpu().numpy(), ci)
+    assert np.array_equal(bits(A.values.cpu().numpy()), bits(va))
+    for b in (8, 16, 24, 32, 7):
+        _check(rp, ci, va, S.uniform_block_ptr(g.n, b))
+
+
+def test_c4_full_size_sampled():
+    """Config C4 at full size: 174x174x22 grid, 1,998,216 rows, skewed hubs,
+    b = 24, in the bench's launch configuration; 400 sampled blocks
+    recomputed by the oracle from rows regenerated on the host."""
+    nx, ny, nz, b = 174, 174, 22, 24
+    g = S.FemGrid(nx, ny, nz)
+    A = bj.synth_fem(nx, ny, nz, 0, g.n)
+    assert A.row_ptr.numel() == g.n + 1
+    bp = S.uniform_block_ptr(g.n, b)
+    bpt = torch.from_numpy(bp).cuda()
+    sizes, vec, val = bj.layout_from_block_ptr(bpt, torch.float64)
+    out = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=torch.float64, device="cuda"))
+    bj.extract(A, bpt, out)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(43)
+    nb = len(bp) - 1
+    hubs = [r // b for r in range(0, g.n, 997) if g.n_extra(r) > 0][:50]
+    ids = np.unique(np.concatenate([rng.choice(nb, 350, replace=False), hubs, [0, nb - 1]]))
+    valh = val.cpu().numpy()
+    got = out.values.cpu().numpy()
+    for i in ids:
+        bs, be = int(bp[i]), int(bp[i + 1])
+        rows = [g.row(r) for r in range(bs, be)]
+        rpl = np.concatenate([[0], np.cumsum([len(c) for c, _ in rows])]).astype(np.int64)
+        ref, sz, _, vl = oracle.extract(rpl, np.concatenate([c for c, _ in rows]),
+                                        np.concatenate([v for _, v in rows]), np.array([0, be - bs], np.int32),
+                                        col_offset=bs)
+        m = be - bs
+        assert np.array_equal(bits(got[valh[i]: valh[i] + m * m]), bits(ref[: m * m]))
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_block_jacobi_handle_setup_apply(dtype):
+    """Row a5 on a FEM slab (local rows, global columns)."""
+    nx, ny, nz = 12, 10, 12
+    g = S.FemGrid(nx, ny, nz)
+    plane = 3 * nx * ny
+    r0, r1 = 3 * plane, 8 * plane
+    A = bj.synth_fem(nx, ny, nz, r0, r1, dtype=dtype)
+    bp = S.uniform_block_ptr(r1 - r0, 24)
+    bpt = torch.from_numpy(bp).cuda()
+    sizes, vec, val = bj.layout_from_block_ptr(bpt, dtype)
+    fac = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=dtype, device="cuda"))
+    piv = torch.empty(r1 - r0, dtype=torch.int32, device="cuda")
+    info = torch.empty(len(bp) - 1, dtype=torch.int32, device="cuda")
+    h = bj.Handle()
+    h.setup(A, bpt, fac, piv, info)
+    x = torch.from_numpy(np.random.default_rng(44).uniform(-1, 1, r1 - r0).astype(NP[dtype])).cuda()
+    y = torch.empty_like(x)
+    h.apply(x, y)
+    torch.cuda.synchronize()
+    rp, ci, va = g.csr(r0, r1, dtype=NP[dtype])
+    D, sz, vo, vl = oracle.extract(rp, ci, va, bp, col_offset=r0)
+    LU, po, io = oracle.getrf_batch(sz, vl, vo, D)
+    yo = oracle.getrs_batch(sz, vl, vo, LU, po, x.cpu().numpy())
+    assert np.array_equal(info.cpu().numpy(), io) and np.array_equal(piv.cpu().numpy(), po)
+    assert np.array_equal(bits(y.cpu().numpy()), bits(yo))
+    # apply twice (stateless) and in place
+    y2 = x.clone()
+    h.apply(y2, y2)
+    torch.cuda.synchronize()
+    assert torch.equal(y2, y)

@@ -1,0 +1,231 @@
+"""GPU parity of GETRF / GETRS (hot-path rows a1, a3, a4) against the CPU
+oracle, through the C ABI.  Bar: pivots, info and block boundaries bit-exact;
+L\\U and x bit-exact under the pinned operation order (R5: explicit FMA, IEEE
+division, ascending k), which implies the north-star tolerances; backward
+error <= 1e-13 (fp64) / 1e-5 (fp32) checked independently."""
+import numpy as np
+import pytest
+import torch
+
+import bj_synth as S
+import oracle
+from gpu_helpers import NP, backward_error, bits, compare_getrf, device_batch, host_layout
+from paper_conf_icpp_anztdfq17_b200 import bj
+
+pytestmark = pytest.mark.gpu
+
+TOL = {torch.float64: 1e-13, torch.float32: 1e-5}
+
+
+def _run(sizes_np, dtype, kind="uniform", values_np=None, plan=True):
+    npdt = NP[dtype]
+    vec, val = host_layout(sizes_np, dtype)
+    A = values_np if values_np is not None else S.block_values(sizes_np, val, dtype=npdt, kind=kind)
+    b = S.rhs_values(sizes_np, dtype=npdt) if len(sizes_np) else np.zeros(0, npdt)
+    batch = device_batch(sizes_np, dtype, values_np=A)
+    # block boundaries (a1) bit-exact
+    assert np.array_equal(batch.vec_off.cpu().numpy(), vec)
+    assert np.array_equal(batch.val_off.cpu().numpy(), val)
+    nvec = int(vec[-1])
+    piv = torch.full((max(nvec, 1),), -7, dtype=torch.int32, device="cuda")
+    info = torch.full((max(len(sizes_np), 1),), -9, dtype=torch.int32, device="cuda")
+    p = bj.Plan(batch.sizes) if plan else None
+    bj.getrf(batch, piv, info, plan=p)
+    bt = torch.from_numpy(b).to("cuda") if nvec else torch.zeros(1, dtype=dtype, device="cuda")
+    x = torch.full_like(bt, float("nan"))
+    bj.getrs(batch, piv, bt, x, plan=p)
+    torch.cuda.synchronize()
+    LU_d = batch.values.cpu().numpy()
+    piv_d = piv.cpu().numpy()[:nvec]
+    info_d = info.cpu().numpy()[: len(sizes_np)]
+    x_d = x.cpu().numpy()[:nvec]
+    LU_o, piv_o, info_o = compare_getrf(sizes_np, val, vec, A, LU_d, piv_d, info_d, dtype)
+    x_o = oracle.getrs_batch(sizes_np, val, vec, LU_o, piv_o, b)
+    return dict(A=A, b=b, vec=vec, val=val, x_d=x_d, x_o=x_o, info=info_d)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_c1_parity(dtype):
+    """Config C1: 1,000 random blocks, m ~ U{4..16}: full oracle comparison."""
+    sizes = S.block_sizes(1000, 4, 16)
+    r = _run(sizes, dtype)
+    assert np.array_equal(bits(r["x_d"]), bits(r["x_o"]))
+    assert backward_error(sizes, r["val"], r["vec"], r["A"], r["b"], r["x_d"]) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("kind", ["uniform", "int"])
+def test_every_order_1_to_32(dtype, kind):
+    """Every m in 1..32, several tiles per warp and a ragged tail per order;
+    'int' blocks (U{-3..3}) have many exact ties and singular steps."""
+    sizes = np.repeat(np.arange(1, 33, dtype=np.int32), 37)
+    rng = np.random.default_rng(5)
+    rng.shuffle(sizes)
+    r = _run(sizes, dtype, kind=kind)
+    if kind == "uniform":
+        assert np.array_equal(bits(r["x_d"]), bits(r["x_o"]))
+        assert backward_error(sizes, r["val"], r["vec"], r["A"], r["b"], r["x_d"]) <= TOL[dtype]
+    else:
+        assert (r["info"] > 0).any()           # singular blocks were exercised
+        ok = r["info"] == 0
+        # nonsingular integer blocks: solutions identical where the oracle's is finite
+        xd, xo = r["x_d"], r["x_o"]
+        fin = np.isfinite(xo)
+        assert np.array_equal(bits(xd[fin]), bits(xo[fin]))
+        assert ok.sum() > 100
+
+
+def test_edge_sizes_empty_invalid_and_transient_plan():
+    sizes = np.array([0, 5, 33, 1, -4, 32, 0, 17, 2, 40], dtype=np.int32)
+    vec, val = host_layout(sizes, torch.float64)
+    A = np.random.default_rng(3).uniform(-1, 1, size=int(val[-1]))
+    r = _run(sizes, torch.float64, values_np=A, plan=False)
+    assert r["info"].tolist()[2] == -1 and r["info"].tolist()[4] == -1 and r["info"].tolist()[9] == -1
+    assert r["info"][0] == 0 and r["info"][6] == 0
+
+
+def test_empty_batch():
+    _run(np.zeros(0, np.int32), torch.float64)
+
+
+def test_special_matrices():
+    """identity, permutation, diagonal, zero, -0 column, NaN/Inf injection."""
+    rng = np.random.default_rng(9)
+    blocks = []
+    m = 8
+    blocks.append(np.eye(m))
+    blocks.append(np.eye(m)[rng.permutation(m)])
+    blocks.append(np.diag(rng.uniform(0.5, 2, m)))
+    blocks.append(np.zeros((m, m)))
+    z = rng.uniform(-1, 1, (m, m)); z[:, 3] = -0.0
+    blocks.append(z)
+    n = rng.uniform(-1, 1, (m, m)); n[2, 4] = np.nan
+    blocks.append(n)
+    f = rng.uniform(-1, 1, (m, m)); f[5, 0] = np.inf
+    blocks.append(f)
+    sizes = np.full(len(blocks), m, np.int32)
+    vec, val = host_layout(sizes, torch.float64)
+    A = np.zeros(int(val[-1]))
+    for i, B in enumerate(blocks):
+        A[val[i]: val[i] + m * m] = B.flatten(order="F")
+    _run(sizes, torch.float64, values_np=A)
+
+
+def test_padding_invariance_on_device():
+    """a k x k block embedded in 32 x 32 (identity padding) gives the
+    same leading factors and pivots on the device as the k x k block."""
+    rng = np.random.default_rng(10)
+    for k in (3, 13, 17, 31):
+        Ak = rng.uniform(-1, 1, (k, k))
+        B = np.eye(32); B[:k, :k] = Ak
+        sizes = np.array([k, 32], np.int32)
+        vec, val = host_layout(sizes, torch.float64)
+        A = np.zeros(int(val[-1]))
+        A[val[0]: val[0] + k * k] = Ak.flatten(order="F")
+        A[val[1]: val[1] + 1024] = B.flatten(order="F")
+        batch = device_batch(sizes, torch.float64, values_np=A)
+        piv = torch.zeros(int(vec[-1]), dtype=torch.int32, device="cuda")
+        info = torch.zeros(2, dtype=torch.int32, device="cuda")
+        bj.getrf(batch, piv, info)
+        LU = batch.values.cpu().numpy()
+        p = piv.cpu().numpy()
+        assert np.array_equal(p[:k], p[k: 2 * k])
+        lead = LU[val[1]: val[1] + 1024].reshape(32, 32, order="F")[:k, :k]
+        assert np.array_equal(bits(lead.copy()), bits(LU[val[0]: val[0] + k * k].reshape(k, k, order="F").copy()))
+
+
+def test_getrs_in_place_alias():
+    sizes = S.block_sizes(500, 1, 32)
+    vec, val = host_layout(sizes, torch.float64)
+    batch = device_batch(sizes, torch.float64)
+    piv = torch.zeros(int(vec[-1]), dtype=torch.int32, device="cuda")
+    info = torch.zeros(len(sizes), dtype=torch.int32, device="cuda")
+    bj.getrf(batch, piv, info)
+    b = torch.from_numpy(S.rhs_values(sizes)).cuda()
+    x = torch.empty_like(b)
+    bj.getrs(batch, piv, b, x)
+    y = b.clone()
+    bj.getrs(batch, piv, y, y)
+    torch.cuda.synchronize()
+    assert torch.equal(x, y)
+
+
+def test_device_generator_matches_host_generator():
+    for dtype in (torch.float64, torch.float32):
+        sizes_d = bj.synth_sizes(5000, 1, 32, first=123)
+        sizes = S.block_sizes(5000, 1, 32, first=123)
+        assert np.array_equal(sizes_d.cpu().numpy(), sizes)
+        vec, val = host_layout(sizes, dtype)
+        for kind, kname in ((0, "uniform"), (1, "int")):
+            batch = device_batch(sizes, dtype, first=123, kind=kind)
+            A = S.block_values(sizes, val, first=123, dtype=NP[dtype], kind=kname)
+            assert np.array_equal(bits(batch.values.cpu().numpy()[: len(A)]), bits(A))
+        rhs = bj.synth_rhs(batch, first=123)
+        assert np.array_equal(bits(rhs.cpu().numpy()[: int(vec[-1])]), bits(S.rhs_values(sizes, first=123,
+                                                                                          dtype=NP[dtype])))
+
+
+def test_gesv_host_end_to_end():
+    """bj_gesv_host (host buffers in/out) equals the oracle."""
+    sizes = S.block_sizes(3000, 4, 32, first=7)
+    vec, val = host_layout(sizes, torch.float64)
+    A = S.block_values(sizes, val, first=7)
+    b = S.rhs_values(sizes, first=7)
+    ws = bj.Workspace()
+    sizes_h = torch.from_numpy(sizes).pin_memory()
+    A_h = torch.from_numpy(A).pin_memory()
+    b_h = torch.from_numpy(b).pin_memory()
+    x_h = torch.empty_like(b_h).pin_memory()
+    piv_h = torch.empty(int(vec[-1]), dtype=torch.int32).pin_memory()
+    info_h = torch.empty(len(sizes), dtype=torch.int32).pin_memory()
+    ws.gesv_host(sizes_h, A_h, b_h, x_h, piv_h, info_h)
+    LU_o, piv_o, info_o = oracle.getrf_batch(sizes, val, vec, A)
+    x_o = oracle.getrs_batch(sizes, val, vec, LU_o, piv_o, b)
+    assert np.array_equal(piv_h.numpy(), piv_o) and np.array_equal(info_h.numpy(), info_o)
+    assert np.array_equal(bits(x_h.numpy()), bits(x_o))
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_c3_full_size_sampled(dtype):
+    """Config C3 at full size (1M blocks, m ~ U{4..32}) in the launch
+    configuration bench.py times; 3,000 sampled blocks recomputed one by one by
+    the oracle from the host generator."""
+    nb = 1_000_000
+    sizes_d = bj.synth_sizes(nb, 4, 32)
+    batch = bj.new_batch(sizes_d, dtype)
+    bj.synth_blocks(batch)
+    b = bj.synth_rhs(batch)
+    plan = bj.Plan(batch.sizes)
+    nvec = int(batch.vec_off[-1].item())
+    piv = torch.empty(nvec, dtype=torch.int32, device="cuda")
+    info = torch.empty(nb, dtype=torch.int32, device="cuda")
+    x = torch.empty_like(b)
+    bj.getrf(batch, piv, info, plan=plan)
+    bj.getrs(batch, piv, b, x, plan=plan)
+    torch.cuda.synchronize()
+    assert int((info != 0).sum().item()) == 0
+    sizes = S.block_sizes(nb, 4, 32)
+    assert np.array_equal(sizes_d.cpu().numpy(), sizes)
+    rng = np.random.default_rng(77)
+    ids = np.unique(np.concatenate([rng.choice(nb, 2998, replace=False), [0, nb - 1]]))
+    vo = batch.val_off.cpu().numpy()
+    ve = batch.vec_off.cpu().numpy()
+    vec_h, val_h = host_layout(sizes, dtype)
+    assert np.array_equal(vo, val_h) and np.array_equal(ve, vec_h)
+    LU_all = batch.values
+    ss = sizes[ids]
+    svec, sval = host_layout(ss, dtype)
+    A_s = S.block_values(ss, sval, dtype=NP[dtype], ids=ids)
+    b_s = S.rhs_values(ss, dtype=NP[dtype], ids=ids)
+    LU_o, piv_o, info_o = oracle.getrf_batch(ss, sval, svec, A_s)
+    x_o = oracle.getrs_batch(ss, sval, svec, LU_o, piv_o, b_s)
+    lu_idx = np.concatenate([np.arange(vo[i], vo[i] + sizes[i] ** 2) for i in ids])
+    v_idx = np.concatenate([np.arange(ve[i], ve[i] + sizes[i]) for i in ids])
+    LU_d = LU_all[torch.from_numpy(lu_idx).cuda()].cpu().numpy()
+    piv_d = piv[torch.from_numpy(v_idx).cuda()].cpu().numpy()
+    x_d = x[torch.from_numpy(v_idx).cuda()].cpu().numpy()
+    LU_o_packed = np.concatenate([LU_o[sval[j]: sval[j] + ss[j] ** 2] for j in range(len(ids))])
+    assert np.array_equal(piv_d, piv_o)
+    assert np.array_equal(bits(LU_d), bits(LU_o_packed))
+    assert np.array_equal(bits(x_d), bits(x_o))
+    assert backward_error(ss, sval, svec, A_s, b_s, x_o) <= TOL[dtype]
