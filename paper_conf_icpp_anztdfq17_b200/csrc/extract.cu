@@ -46,9 +46,9 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
         const int bs = __ldg(block_ptr + b), be = __ldg(block_ptr + b + 1);
         const int m = be - bs;
         if (m <= 0 || m > kMaxM) continue;                     // nothing to write / invalid order
-        // lane j <= m holds row_ptr[bs + j]
-        const int64_t rpv = lane <= m ? __ldg(row_ptr + bs + lane) : 0;
-        const int64_t e0 = __shfl_sync(kFull, rpv, 0), e1 = __shfl_sync(kFull, rpv, m);
+        // lane j < m holds row_ptr[bs + j]; every lane holds row_ptr[be]
+        const int64_t rpv = lane < m ? __ldg(row_ptr + bs + lane) : 0;
+        const int64_t e0 = __shfl_sync(kFull, rpv, 0), e1 = __ldg(row_ptr + be);
         if (e1 - e0 > kHeavy) {
             if (lane == 0) heavy[atomicAdd(nheavy, 1ull)] = (int32_t)b;
             continue;
@@ -59,7 +59,9 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
         __syncwarp();
         const int64_t cb = (int64_t)bs + col_offset, ce = (int64_t)be + col_offset;
         for (int r = 0; r < m; ++r) {
-            const int64_t rs = __shfl_sync(kFull, rpv, r), re = __shfl_sync(kFull, rpv, r + 1);
+            const int64_t rs = __shfl_sync(kFull, rpv, r);
+            const int64_t rn = __shfl_sync(kFull, rpv, (r + 1) & 31);
+            const int64_t re = r + 1 < m ? rn : e1;
             for (int64_t e = rs + lane; e < re; e += 32) {
                 const int64_t c = __ldg(col_idx + e);
                 if (c >= cb && c < ce) T[r + (int)(c - cb) * m] = __ldg(values + e);

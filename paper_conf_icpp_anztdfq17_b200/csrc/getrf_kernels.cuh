@@ -12,11 +12,15 @@
 //    no lane computes on padding (the reference pads to 32);
 //  * the code is fully specialised on m (unrolled k and j loops), so the
 //    register indices are static;
-//  * pivot search: unsigned max over the |a| bit patterns (+1 for candidates,
-//    0 for pivoted rows) within the tile, lowest lane among the maxima via a
-//    ballot -> exactly the oracle's tie rule (R1, R2);
+//  * pivot search: unsigned max (REDUX for a full warp) over the high word of
+//    |a| (bit 31 set for candidates, 0 for pivoted rows) within the tile, lowest
+//    lane among the maxima via a ballot; high-word ties are resolved on the low
+//    word -> exactly the oracle's order and tie rule (R1, R2);
 //  * implicit pivoting: a per-lane tag (step at which the row was pivoted);
-//    the pivot row is broadcast, never swapped;
+//    the pivot row is never swapped: its lane publishes its trailing part to a
+//    per-warp smem buffer (16-B stores) and the unpivoted lanes read it back
+//    as 16-B broadcasts inside a divergent branch, so pivoted rows need no
+//    selects;
 //  * combined row swap at write-back: lane r stores its row at position
 //    tag-1 of every column (a permutation inside each column -> coalesced),
 //    and the permutation vector perm[tag-1] = r.
@@ -31,10 +35,8 @@ template <typename R, int M>
 __device__ __forceinline__ void getrf_tile(R *__restrict__ A, const int64_t *__restrict__ val_off,
                                            const int64_t *__restrict__ vec_off, int32_t *__restrict__ piv,
                                            int32_t *__restrict__ info, const int32_t *__restrict__ order,
-                                           int64_t first, int64_t last) {
-    using Key = typename Num<R>::Key;
+                                           int64_t first, int64_t last, R *__restrict__ wbuf) {
     constexpr int T = tile_width(M);
-    constexpr unsigned TMASK = (T == 32) ? kFull : ((1u << (T & 31)) - 1u);
     const int lane = threadIdx.x & 31;
     const int t = lane / T;
     const int r = lane % T;
@@ -44,6 +46,7 @@ __device__ __forceinline__ void getrf_tile(R *__restrict__ A, const int64_t *__r
     const int blk = tile_ok ? __ldg(order + idx) : 0;
     const bool row_ok = tile_ok && (r < M);
     R *Ab = A + (tile_ok ? __ldg(val_off + blk) : 0);
+    R *buf = wbuf + tbase;                 // this tile's pivot-row buffer (T elements, smem)
 
     // Load row r (column-major: lanes of a tile read consecutive addresses).
     R a[M];
@@ -56,28 +59,73 @@ __device__ __forceinline__ void getrf_tile(R *__restrict__ A, const int64_t *__r
     int inf = 0;
     static_for<0, M>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
-        // lines 5-7 of Fig. 1 bottom: max |a_ik| over the unpivoted rows.
-        const Key key = (tag == 0) ? Key(Num<R>::absbits(a[k]) + 1) : Key(0);
-        Key kmax = key;
-#pragma unroll
-        for (int off = T / 2; off >= 1; off >>= 1) {
-            const Key o = __shfl_xor_sync(kFull, kmax, off);
-            kmax = o > kmax ? o : kmax;
+        // Fig. 1 bottom lines 5-7: max |a_ik| over the unpivoted rows.  Key =
+        // high word of |a| with bit 31 set for candidates (0 for pivoted rows);
+        // exact ties of the high word (or |a| < 2^-1022) are resolved on the low
+        // word in a rare second pass, so the order is exactly the oracle's.
+        const unsigned key = (tag == 0) ? (Num<R>::key_hi(a[k]) | 0x80000000u) : 0u;
+        const unsigned kmax = tile_max<T>(key);
+        unsigned tb = tile_bits<T>(__ballot_sync(kFull, key == kmax), tbase);
+        bool sing;
+        if constexpr (sizeof(R) == 8) {
+            const bool amb = (__popc(tb) > 1) || (kmax == 0x80000000u);
+            sing = false;
+            if (__any_sync(kFull, amb)) {
+                const bool cand = (key == kmax);
+                const unsigned lo = cand ? Num<R>::key_lo(a[k]) : 0u;
+                const unsigned lmax = tile_max<T>(lo);
+                tb = tile_bits<T>(__ballot_sync(kFull, cand && lo == lmax), tbase);
+                sing = (kmax == 0x80000000u) && (lmax == 0u);
+            }
+        } else {
+            sing = (kmax == 0x80000000u);
         }
-        const unsigned ball = __ballot_sync(kFull, key == kmax);
-        const unsigned tb = (T == 32) ? ball : ((ball >> tbase) & TMASK);
-        const int ipiv = __ffs(tb) - 1;                 // lowest row among the maxima
-        const bool sing = (kmax == Key(1));             // all candidates are +-0 (R4)
-        if (r == ipiv) tag = k + 1;                     // line 9: p(ipiv) = k
-        const R d = __shfl_sync(kFull, a[k], tbase + ipiv);   // line 12
-        const bool upd = (tag == 0) && !sing;
-        if (upd) a[k] = Num<R>::div(a[k], d);           // line 13: SCAL
-        static_for<k + 1, M>([&](auto jc) {             // lines 14-15: GER
-            constexpr int j = decltype(jc)::value;
-            const R u = __shfl_sync(kFull, a[j], tbase + ipiv);
-            if (upd) a[j] = Num<R>::fma(-a[k], u, a[j]);
-        });
+        const int ipiv = __ffs(tb) - 1;                 // lowest row among the maxima (R1)
+        if (r == ipiv) {                                // line 9: p(ipiv) = k; publish the pivot row
+            tag = k + 1;
+            if constexpr (sizeof(R) == 8 && T > 1) {
+                constexpr int j0 = k & ~1;
+                static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
+                    constexpr int j = j0 + 2 * decltype(pc)::value;
+                    if constexpr (j + 1 < M) *reinterpret_cast<double2 *>(buf + j) = make_double2(a[j], a[j + 1]);
+                    else buf[j] = a[j];
+                });
+            } else {
+                static_for<k, M>([&](auto jc) {
+                    constexpr int j = decltype(jc)::value;
+                    buf[j] = a[j];
+                });
+            }
+        }
+        __syncwarp();
+        const R d = buf[k];                             // line 12
+        if (tag == 0 && !sing) {                        // lines 13-15 on the unpivoted rows
+            const R l = Num<R>::div(a[k], d);           // SCAL (IEEE division)
+            a[k] = l;
+            if constexpr (sizeof(R) == 8) {             // GER, pivot row read as 16-B pairs
+                if constexpr ((k + 1) & 1) {
+                    a[k + 1] = Num<R>::fma(-l, buf[k + 1], a[k + 1]);
+                }
+                constexpr int j0 = (k + 2) & ~1;
+                static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
+                    constexpr int j = j0 + 2 * decltype(pc)::value;
+                    if constexpr (j + 1 < M) {
+                        const double2 u = *reinterpret_cast<const double2 *>(buf + j);
+                        a[j] = Num<R>::fma(-l, u.x, a[j]);
+                        a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
+                    } else {
+                        a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                    }
+                });
+            } else {
+                static_for<k + 1, M>([&](auto jc) {
+                    constexpr int j = decltype(jc)::value;
+                    a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                });
+            }
+        }
         if (sing && inf == 0) inf = k + 1;
+        __syncwarp();
     });
     // lines 18-19: combined row swap while off-loading L\U.
     if (row_ok) {
@@ -94,23 +142,25 @@ __device__ __forceinline__ void getrf_tile(R *__restrict__ A, const int64_t *__r
 template <typename R, int M, int MHI>
 __device__ __forceinline__ void getrf_dispatch(int m, R *A, const int64_t *val_off, const int64_t *vec_off,
                                                int32_t *piv, int32_t *info, const int32_t *order,
-                                               int64_t first, int64_t last) {
+                                               int64_t first, int64_t last, R *wbuf) {
     if (m == M) {
-        getrf_tile<R, M>(A, val_off, vec_off, piv, info, order, first, last);
+        getrf_tile<R, M>(A, val_off, vec_off, piv, info, order, first, last, wbuf);
     } else {
-        if constexpr (M < MHI) getrf_dispatch<R, M + 1, MHI>(m, A, val_off, vec_off, piv, info, order, first, last);
+        if constexpr (M < MHI)
+            getrf_dispatch<R, M + 1, MHI>(m, A, val_off, vec_off, piv, info, order, first, last, wbuf);
     }
 }
 
 // One size class [MLO, MHI].  Tasks are enumerated bin by bin (all tasks of
 // order MLO first); warp w takes tasks w, w + nwarps, ...
 template <typename R, int MLO, int MHI>
-__global__ void __launch_bounds__(kGetrfThreads)
+__global__ void __launch_bounds__(kGetrfThreads, 4)
 k_getrf_class(R *A, const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off,
               int32_t *__restrict__ piv, int32_t *__restrict__ info, const int32_t *__restrict__ order,
               const int64_t *__restrict__ bin_start) {
     constexpr int NM = MHI - MLO + 1;
     __shared__ int64_t s_pref[NM + 1], s_first[NM], s_last[NM];
+    __shared__ __align__(16) R s_buf[kGetrfThreads];          // 32 elements per warp
     if (threadIdx.x == 0) {
         int64_t acc = 0;
         for (int i = 0; i < NM; ++i) {
@@ -132,7 +182,8 @@ k_getrf_class(R *A, const int64_t *__restrict__ val_off, const int64_t *__restri
         while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
         const int m = MLO + i;
         const int64_t first = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m);
-        getrf_dispatch<R, MLO, MHI>(m, A, val_off, vec_off, piv, info, order, first, s_last[i]);
+        getrf_dispatch<R, MLO, MHI>(m, A, val_off, vec_off, piv, info, order, first, s_last[i],
+                                    s_buf + (threadIdx.x & ~31));
     }
 }
 

@@ -22,6 +22,10 @@ __device__ __forceinline__ void getrs_tile(const R *__restrict__ LU, const int32
         constexpr int j = decltype(jc)::value;
         a[j] = row_ok ? __ldg(LU + r + j * M) : R(0);
     });
+    // U(r,r) again (same cache lines) so lane r can refine 1/U(r,r) off the
+    // critical path; the quotient itself is still the IEEE one (Num::div_pre).
+    const R dg = row_ok ? __ldg(LU + r + r * M) : R(1);
+    const R yrcp = Num<R>::rcp_refine(dg);
     // b := P b: lane r receives b[perm[r]].
     R y = row_ok ? b[__ldg(piv + r)] : R(0);
 
@@ -29,14 +33,14 @@ __device__ __forceinline__ void getrs_tile(const R *__restrict__ LU, const int32
     static_for<0, M - 1>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
         const R yk = __shfl_sync(kFull, y, tbase + k);
-        if (r > k) y = Num<R>::fma(-a[k], yk, y);
+        Num<R>::pfma(r > k, y, -a[k], yk);
     });
     // U x = y, eager and mirrored (R8): y_k /= U(k,k); y_i -= U(i,k) y_k, i < k.
     static_for<0, M>([&](auto kk) {
         constexpr int k = M - 1 - decltype(kk)::value;
-        if (r == k) y = Num<R>::div(y, a[k]);
+        if (r == k) y = Num<R>::div_pre(y, dg, yrcp);
         const R yk = __shfl_sync(kFull, y, tbase + k);
-        if (r < k) y = Num<R>::fma(-a[k], yk, y);
+        Num<R>::pfma(r < k, y, -a[k], yk);
     });
     __syncwarp();                               // every lane has read b before x is written (x may alias b)
     if (row_ok) x[r] = y;

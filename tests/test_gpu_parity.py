@@ -21,7 +21,7 @@ def _run(sizes_np, dtype, kind="uniform", values_np=None, plan=True):
     npdt = NP[dtype]
     vec, val = host_layout(sizes_np, dtype)
     A = values_np if values_np is not None else S.block_values(sizes_np, val, dtype=npdt, kind=kind)
-    b = S.rhs_values(sizes_np, dtype=npdt) if len(sizes_np) else np.zeros(0, npdt)
+    b = S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt) if len(sizes_np) else np.zeros(0, npdt)
     batch = device_batch(sizes_np, dtype, values_np=A)
     # block boundaries (a1) bit-exact
     assert np.array_equal(batch.vec_off.cpu().numpy(), vec)
