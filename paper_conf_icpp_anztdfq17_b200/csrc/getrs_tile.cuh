@@ -30,16 +30,18 @@ __device__ __forceinline__ void getrs_tile(const R *__restrict__ LU, const int32
     R y = row_ok ? b[__ldg(piv + r)] : R(0);
 
     // L y = P b, eager (Fig. 2 bottom): y_i -= L(i,k) y_k for i > k.
+    // (T == 32: the source lane is a compile-time constant -> the cheap
+    // warp-uniform SHFL; sub-warp tiles need per-tile sources.)
     static_for<0, M - 1>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
-        const R yk = __shfl_sync(kFull, y, tbase + k);
+        const R yk = (T == 32) ? __shfl_sync(kFull, y, k) : __shfl_sync(kFull, y, tbase + k);
         Num<R>::pfma(r > k, y, -a[k], yk);
     });
     // U x = y, eager and mirrored (R8): y_k /= U(k,k); y_i -= U(i,k) y_k, i < k.
     static_for<0, M>([&](auto kk) {
         constexpr int k = M - 1 - decltype(kk)::value;
         if (r == k) y = Num<R>::div_pre(y, dg, yrcp);
-        const R yk = __shfl_sync(kFull, y, tbase + k);
+        const R yk = (T == 32) ? __shfl_sync(kFull, y, k) : __shfl_sync(kFull, y, tbase + k);
         Num<R>::pfma(r < k, y, -a[k], yk);
     });
     __syncwarp();                               // every lane has read b before x is written (x may alias b)

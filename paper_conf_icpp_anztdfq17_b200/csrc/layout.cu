@@ -81,36 +81,41 @@ k_plan_hist(const int32_t *__restrict__ sizes, int64_t n, int64_t *__restrict__ 
     for (int b = threadIdx.x; b < kBins; b += blockDim.x) hist[(int64_t)blockIdx.x * kBins + b] = cnt[b];
 }
 
-// Single CTA: hist[tile][bin] -> absolute start of (tile, bin) in `order`;
-// bin_start[bin] = start of bin (bin_start[kBins] = n).
-__global__ void __launch_bounds__(64) k_plan_offsets(int64_t *hist, int64_t ntiles, int64_t *bin_start) {
+// Single CTA, one warp per bin: exclusive scan of hist[.][bin] over the tiles
+// (warp-wide chunks of 32), then bin starts; hist becomes the absolute start
+// of (tile, bin) in `order`.
+__global__ void __launch_bounds__(1024) k_plan_offsets(int64_t *hist, int64_t ntiles, int64_t *bin_start) {
     __shared__ int64_t tot[kBins];
-    const int b = threadIdx.x;
-    int64_t acc = 0;
-    if (b < kBins) {
-        for (int64_t t = 0; t < ntiles; ++t) {
-            int64_t c = hist[t * kBins + b];
-            hist[t * kBins + b] = acc;
-            acc += c;
+    __shared__ int64_t base[kBins + 1];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int b = w; b < kBins; b += nw) {
+        int64_t carry = 0;
+        for (int64_t t0 = 0; t0 < ntiles; t0 += 32) {
+            const int64_t t = t0 + lane;
+            const int64_t c = t < ntiles ? hist[t * kBins + b] : 0;
+            int64_t inc = c;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const int64_t v = __shfl_up_sync(kFull, inc, off);
+                if (lane >= off) inc += v;
+            }
+            if (t < ntiles) hist[t * kBins + b] = carry + inc - c;
+            carry += __shfl_sync(kFull, inc, 31);
         }
-        tot[b] = acc;
+        if (lane == 0) tot[b] = carry;
     }
     __syncthreads();
-    if (b == 0) {
+    if (threadIdx.x == 0) {
         int64_t s = 0;
         for (int i = 0; i < kBins; ++i) {
-            int64_t c = tot[i];
-            tot[i] = s;
+            base[i] = s;
             bin_start[i] = s;
-            s += c;
+            s += tot[i];
         }
         bin_start[kBins] = s;
     }
     __syncthreads();
-    if (b < kBins) {
-        const int64_t s = tot[b];
-        for (int64_t t = 0; t < ntiles; ++t) hist[t * kBins + b] += s;
-    }
+    for (int64_t i = threadIdx.x; i < ntiles * kBins; i += blockDim.x) hist[i] += base[i % kBins];
 }
 
 __global__ void __launch_bounds__(kPlanThreads)
@@ -161,7 +166,7 @@ bj_status build_plan(int64_t nb, const int32_t *sizes, int32_t *order, int64_t *
     BJ_CUDA_TRY(cudaMallocAsync((void **)&hist, sizeof(int64_t) * kBins * ntiles, s));
     k_plan_hist<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist);
     BJ_LAUNCH_CHECK();
-    k_plan_offsets<<<1, 64, 0, s>>>(hist, ntiles, bin_start);
+    k_plan_offsets<<<1, 1024, 0, s>>>(hist, ntiles, bin_start);
     BJ_LAUNCH_CHECK();
     k_plan_scatter<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist, order);
     BJ_LAUNCH_CHECK();
