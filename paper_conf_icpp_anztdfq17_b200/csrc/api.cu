@@ -161,9 +161,11 @@ bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, co
         p = &tmp;
     }
     if (blocks->dtype == BJ_F64)
-        st = getrf_run<double>((double *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(), s);
+        st = getrf_run<double>((double *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                               blocks->sizes, s);
     else
-        st = getrf_run<float>((float *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(), s);
+        st = getrf_run<float>((float *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                              blocks->sizes, s);
     if (!plan) plan_free_async(&tmp, s);
     return st;
 }

@@ -1,14 +1,13 @@
 // getrf.cu -- host driver of hot-path row a3 (kernels: getrf_kernels.cuh,
 // instantiated per (dtype, size class) in getrf_inst.cu so they compile in
 // parallel).
-#include "common.cuh"
-#include "internal.h"
+#include "getrf_fast.cuh"
 
 namespace bj {
 
 template <typename R, int MLO, int MHI>
-bj_status launch_getrf_class(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
-                             const PlanView &p, cudaStream_t s);
+bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
+                            const PlanView &p, int32_t *safe_list, unsigned *safe_count, cudaStream_t s);
 
 // info for blocks of order 0 (nothing to factor) and of invalid order (-1).
 __global__ void k_info_trivial(int32_t *__restrict__ info, const int32_t *__restrict__ order,
@@ -24,21 +23,29 @@ __global__ void k_info_trivial(int32_t *__restrict__ info, const int32_t *__rest
 
 template <typename R>
 bj_status getrf_run(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
-                    const PlanView &p, cudaStream_t s) {
+                    const PlanView &p, const int32_t *sizes, cudaStream_t s) {
     if (p.nblocks == 0) return BJ_OK;
+    char *scratch = nullptr;
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch, 16 + sizeof(int32_t) * (size_t)p.nblocks, s));
+    unsigned *safe_count = reinterpret_cast<unsigned *>(scratch);
+    int32_t *safe_list = reinterpret_cast<int32_t *>(scratch + 16);
+    BJ_CUDA_TRY(cudaMemsetAsync(safe_count, 0, sizeof(unsigned), s));
     bj_status st;
-    if ((st = launch_getrf_class<R, 17, 32>(A, val_off, vec_off, piv, info, p, s)) != BJ_OK) return st;
-    if ((st = launch_getrf_class<R, 9, 16>(A, val_off, vec_off, piv, info, p, s)) != BJ_OK) return st;
-    if ((st = launch_getrf_class<R, 5, 8>(A, val_off, vec_off, piv, info, p, s)) != BJ_OK) return st;
-    if ((st = launch_getrf_class<R, 1, 4>(A, val_off, vec_off, piv, info, p, s)) != BJ_OK) return st;
+    if ((st = launch_getrf_fast<R, 17, 32>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    if ((st = launch_getrf_fast<R, 9, 16>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    if ((st = launch_getrf_fast<R, 5, 8>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    if ((st = launch_getrf_fast<R, 1, 4>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    k_getrf_safe<R><<<sm_count() * 2, 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info, safe_list, safe_count);
+    BJ_LAUNCH_CHECK();
     k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
     BJ_LAUNCH_CHECK();
+    BJ_CUDA_TRY(cudaFreeAsync(scratch, s));
     return BJ_OK;
 }
 
 template bj_status getrf_run<double>(double *, const int64_t *, const int64_t *, int32_t *, int32_t *,
-                                     const PlanView &, cudaStream_t);
+                                     const PlanView &, const int32_t *, cudaStream_t);
 template bj_status getrf_run<float>(float *, const int64_t *, const int64_t *, int32_t *, int32_t *,
-                                    const PlanView &, cudaStream_t);
+                                    const PlanView &, const int32_t *, cudaStream_t);
 
 }  // namespace bj

@@ -6,6 +6,7 @@
 #include <vector>
 #include <algorithm>
 #include "getrf_kernels.cuh"
+#include "getrf_fast.cuh"
 
 namespace bj {
 void count_launch(int) {}
@@ -68,6 +69,82 @@ void run_mix(int64_t nb, const char *name) {
     cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
 }
 
+template <int LO, int HI, int F>
+void run_mix_fast(int64_t nb, const char *name) {
+    std::vector<int64_t> vo(nb + 1), ve(nb + 1);
+    std::vector<int32_t> ord(nb), sz(nb);
+    std::vector<int64_t> cnt(kBins + 1, 0);
+    std::vector<int> m_of(nb);
+    for (int64_t i = 0; i < nb; ++i) m_of[i] = LO + (int)((i * (HI - LO + 1)) / nb);
+    vo[0] = 0; ve[0] = 0;
+    for (int64_t i = 0; i < nb; ++i) { int m = m_of[i]; sz[i] = m; vo[i + 1] = vo[i] + (m * m + 1) / 2 * 2; ve[i + 1] = ve[i] + m; ord[i] = (int32_t)i; cnt[m]++; }
+    std::vector<int64_t> bs(kBins + 1, 0);
+    int64_t acc = 0;
+    for (int b = 0; b < kBins; ++b) { bs[b] = acc; acc += cnt[b]; }
+    bs[kBins] = acc;
+    double *A, *A0; int64_t *dvo, *dve, *dbs; int32_t *dord, *piv, *info, *list, *dsz; unsigned *count;
+    const int64_t tot = vo[nb];
+    cudaMalloc(&A, tot * 8); cudaMalloc(&A0, tot * 8);
+    cudaMalloc(&dvo, (nb + 1) * 8); cudaMalloc(&dve, (nb + 1) * 8); cudaMalloc(&dbs, (kBins + 1) * 8);
+    cudaMalloc(&dord, nb * 4); cudaMalloc(&piv, ve[nb] * 4); cudaMalloc(&info, nb * 4); cudaMalloc(&list, nb * 4);
+    cudaMalloc(&count, 4); cudaMalloc(&dsz, nb * 4);
+    cudaMemcpy(dvo, vo.data(), (nb + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dve, ve.data(), (nb + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dbs, bs.data(), (kBins + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dord, ord.data(), nb * 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(dsz, sz.data(), nb * 4, cudaMemcpyHostToDevice);
+    fill<<<1024, 256>>>(A0, tot, 12345);
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrf_fast<double, LO, HI, F>, kFastThreads, 0);
+    const int grid = per_sm * sm_count();
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    std::vector<float> ts;
+    unsigned hc = 0;
+    for (int rep = 0; rep < 5; ++rep) {
+        cudaMemcpy(A, A0, tot * 8, cudaMemcpyDeviceToDevice);
+        cudaMemset(count, 0, 4);
+        cudaEventRecord(e0);
+        k_getrf_fast<double, LO, HI, F><<<grid, kFastThreads>>>(A, dvo, dve, piv, info, dord, dbs, list, count);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        if (rep) ts.push_back(ms);
+        cudaMemcpy(&hc, count, 4, cudaMemcpyDeviceToHost);
+    }
+    std::sort(ts.begin(), ts.end());
+    double bytes = 0;
+    for (int64_t i = 0; i < nb; ++i) bytes += 2.0 * 8 * m_of[i] * m_of[i] + 4 * m_of[i] + 20;
+    printf("%-26s M=%2d..%2d  occ=%d/SM  %8.1f us  %7.1f GB/s  %6.1f Mblk/s  deferred=%u err=%s\n", name, LO, HI, per_sm * 4,
+           ts[0] * 1e3, bytes / (ts[0] * 1e-3) / 1e9, nb / (ts[0] * 1e-3) / 1e6, hc, cudaGetErrorString(cudaGetLastError()));
+    cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
+    cudaFree(list); cudaFree(count); cudaFree(dsz);
+}
+
+template <int M>
+void run_fast1(int64_t nb, const char *name) {
+    const int64_t per = (M * M + 1) / 2 * 2;
+    std::vector<int64_t> vo(nb + 1), ve(nb + 1); std::vector<int32_t> ord(nb);
+    for (int64_t i = 0; i <= nb; ++i) { vo[i] = i * per; ve[i] = i * M; }
+    for (int64_t i = 0; i < nb; ++i) ord[i] = (int32_t)i;
+    std::vector<int64_t> bs(kBins + 1); for (int b = 0; b <= kBins; ++b) bs[b] = b <= M ? 0 : nb;
+    double *A; int64_t *dvo, *dve, *dbs; int32_t *dord, *piv, *info, *list; unsigned *count;
+    cudaMalloc(&A, per * nb * 8); cudaMalloc(&dvo, (nb + 1) * 8); cudaMalloc(&dve, (nb + 1) * 8); cudaMalloc(&dbs, (kBins + 1) * 8);
+    cudaMalloc(&dord, nb * 4); cudaMalloc(&piv, nb * M * 4); cudaMalloc(&info, nb * 4); cudaMalloc(&list, nb * 4); cudaMalloc(&count, 4);
+    cudaMemcpy(dvo, vo.data(), (nb + 1) * 8, cudaMemcpyHostToDevice); cudaMemcpy(dve, ve.data(), (nb + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dbs, bs.data(), (kBins + 1) * 8, cudaMemcpyHostToDevice); cudaMemcpy(dord, ord.data(), nb * 4, cudaMemcpyHostToDevice);
+    fill<<<1024, 256>>>(A, per * nb, 777); cudaMemset(count, 0, 4);
+    k_getrf_fast<double, M, M, 0><<<sm_count(), 32>>>(A, dvo, dve, piv, info, dord, dbs, list, count);
+    cudaDeviceSynchronize();
+#ifdef BJ_TRACE
+    long long t[64]; cudaMemcpyFromSymbol(t, g_ftrace, sizeof(t));
+#else
+    long long t[64] = {0};
+#endif
+    printf("%s M=%d per-step cycles:", name, M);
+    for (int k = 0; k + 1 < M; ++k) printf(" %lld", t[k + 1] - t[k]);
+    printf("\n");
+}
+
 template <int M, int V>
 void run(int64_t nb, const char *name, int force_warps_per_sm = 0) {
     const int64_t per = (M * M + 1) / 2 * 2;
@@ -112,14 +189,21 @@ void run(int64_t nb, const char *name, int force_warps_per_sm = 0) {
 }
 
 int main() {
-    run<32, 32>(148, "trace 1 block/SM", 1);
-    long long t[64];
-    cudaMemcpyFromSymbol(t, g_trace, sizeof(t));
-    printf("load: %lld cycles\n", t[1] - t[0]);
-    for (int k = 0; k < 32; ++k) printf("step %2d: %lld\n", k, (k < 31 ? t[3 + k] : t[1]) - t[2 + k]);
-    run<32, 32>(148 * 4, "trace 4 blocks/warp", 1);
-    cudaMemcpyFromSymbol(t, g_trace, sizeof(t));
-    printf("load: %lld cycles\n", t[1] - t[0]);
-    for (int k = 0; k < 31; ++k) printf("step %2d: %lld\n", k, t[3 + k] - t[2 + k]);
+#ifdef BJ_TRACE
+    run_fast1<32>(148, "FAST 1 warp");
+    run_fast1<24>(148, "FAST 1 warp");
+    run_fast1<16>(296, "FAST 1 warp");
+#else
+    run_mix<17, 32, 0>(552000, "mix smem base (old)");
+    run_mix_fast<17, 32, 0>(552000, "mix FAST F0 smem");
+    run_mix_fast<17, 32, 1>(552000, "mix FAST F1 shfl");
+    run_mix_fast<17, 32, 2>(552000, "mix FAST F2 smem+pre");
+    run_mix<9, 16, 0>(276000, "mix9-16 old");
+    run_mix_fast<9, 16, 0>(276000, "mix9-16 FAST F0");
+    run_mix_fast<9, 16, 2>(276000, "mix9-16 FAST F2");
+    run_mix<5, 8, 0>(138000, "mix5-8 old");
+    run_mix_fast<5, 8, 0>(138000, "mix5-8 FAST F0");
+    run_mix_fast<1, 4, 0>(69000, "mix1-4 FAST F0");
+#endif
     return 0;
 }
