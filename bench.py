@@ -31,12 +31,16 @@ import torch.distributed as dist
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22)}   # per-GPU z-slab of 22 planes
+
 CONFIGS = {
     # name: (nblocks per GPU, lo, hi, dtype, description)
     "C3": (1_000_000, 4, 32, torch.float64, "C3: 1M blocks/GPU, m ~ U{4..32}, fp64, LU + solve"),
     "C3f32": (1_000_000, 4, 32, torch.float32, "C3: 1M blocks/GPU, m ~ U{4..32}, fp32, LU + solve"),
     "C2": (40_000, 32, 32, torch.float64, "C2: 40,000 blocks 32x32/GPU, fp64, LU + solve"),
     "C1": (1_000, 4, 16, torch.float64, "C1: 1,000 blocks m ~ U{4..16}, fp64 (latency case, L2-resident)"),
+    "C4": (0, 24, 24, torch.float64, "C4: diagonal-block extraction, 27-pt x 3-dof FEM CSR, 1,998,216 rows/GPU, skewed hubs"),
+    "C5": (0, 24, 24, torch.float64, "C5: block-Jacobi setup (extract + getrf) + 100 applies, 1,998,216 rows/GPU, b = 24"),
 }
 
 
@@ -211,10 +215,10 @@ def run_ours(args, ws, rank, local):
         nb_per = args.nblocks
     nb_total = nb_per * ws
     # --- partition (row a6): global sizes from the counter generator
+    from paper_conf_icpp_anztdfq17_b200 import dist as D
     sizes_all = bj.synth_sizes(nb_total, lo, hi)
     sizes_h = sizes_all.cpu().numpy()
-    bounds = bj.partition(sizes_h, ws)
-    first, last = int(bounds[rank]), int(bounds[rank + 1])
+    first, last = D.shard(sizes_h, ws, rank)
     nb = last - first
     sizes = sizes_all[first:last].clone()
     del sizes_all
@@ -376,6 +380,100 @@ def run_ours(args, ws, rank, local):
         print(json.dumps(line), flush=True)
 
 
+def run_fem(args, ws, rank, local):
+    """C4 (extraction) and C5 (setup + 100 applies) on a per-rank z-slab of a
+    174 x 174 x (22 * ws) node grid (rows sharded; global column ids)."""
+    from paper_conf_icpp_anztdfq17_b200 import bj
+    nx, ny, nzr = FEM[args.config]
+    b = args.block or 24
+    dt = torch.float64
+    nz = nzr * ws
+    plane = 3 * nx * ny
+    r0, r1 = rank * nzr * plane, (rank + 1) * nzr * plane
+    n = r1 - r0
+    A = bj.synth_fem(nx, ny, nz, r0, r1, dtype=dt)
+    bp = torch.arange(0, n + b, b, dtype=torch.int32, device="cuda").clamp_(max=n)
+    bp = torch.unique_consecutive(bp)
+    nb = bp.numel() - 1
+    sizes, vec, val = bj.layout_from_block_ptr(bp, dt)
+    out = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=dt, device="cuda"))
+    # algorithmic bytes (SURVEY 8(d))
+    rows = torch.repeat_interleave(torch.arange(n, device="cuda"), A.row_ptr.diff())
+    blk_of_row = torch.div(rows, b, rounding_mode="floor")
+    c = A.col_idx.long() - r0
+    hits = int(((c >= blk_of_row * b) & (c < torch.clamp((blk_of_row + 1) * b, max=n))).sum().item())
+    del rows, blk_of_row, c
+    m = sizes.long()
+    ext_bytes = 8 * (n + 1) + 4 * A.col_idx.numel() + 8 * hits + 8 * int((m * m).sum().item()) + 4 * (nb + 1)
+    getrf_bytes = int((2 * 8 * m * m + 4 * m + 20).sum().item())
+    getrs_bytes = int((8 * m * m + 4 * m + 16 * m + 16).sum().item())
+    stream = torch.cuda.current_stream()
+    hbm, peak_src = load_peaks()
+    piv = torch.empty(n, dtype=torch.int32, device="cuda")
+    info = torch.empty(nb, dtype=torch.int32, device="cuda")
+    x = torch.rand(n, dtype=dt, device="cuda") * 2 - 1
+    y = torch.empty_like(x)
+    h = bj.Handle() if args.config == "C5" else None
+    napply = 100
+
+    def step(evs=None):
+        if args.config == "C4":
+            bj.extract(A, bp, out)
+        else:
+            if evs is not None:
+                evs[0].record(stream)
+            h.setup(A, bp, out, piv, info)
+            if evs is not None:
+                evs[1].record(stream)
+            for _ in range(napply):
+                h.apply(x, y)
+
+    for _ in range(args.warmup):
+        step()
+    barrier(ws)
+    sampler = ClockSampler(local)
+    bj.launch_count_reset()
+    with sampler:
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+        barrier(ws)
+        e0.record(stream)
+        for i in range(args.steps):
+            step(evs[i] if args.config == "C5" else None)
+        e1.record(stream)
+        barrier(ws)
+    launches = bj.launch_count()
+    t_ms = max_over_ranks(e0.elapsed_time(e1), ws)
+    ms = t_ms / args.steps
+    line = {"n_gpus": ws, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic (counter-based FEM CSR generated on device)",
+            "gpu_launches": launches, "clocks": sampler.summary()}
+    if args.config == "C4":
+        achieved = ext_bytes / (ms * 1e-3) / 1e9
+        line.update({"metric": "diagonal blocks extracted per second", "value": nb * ws / (ms * 1e-3),
+                     "unit": "blocks/s", "higher_is_better": True,
+                     "config": {"workload": CONFIGS["C4"][4], "block": b, "rows_per_gpu": n, "nnz_per_gpu": A.col_idx.numel(),
+                                "in_block_hits": hits, "l2": "inputs (1.2 GB) larger than L2"},
+                     "roofline": {"bound": "hbm", "kernel": "bj_extract", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                                  "frac": achieved / hbm, "traffic": None, "peak_source": peak_src,
+                                  "bytes_per_launch": ext_bytes}})
+    else:
+        setup_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
+        apply_ms = (ms - setup_ms) / napply
+        line.update({"metric": "block-Jacobi setup + 100 applies per second", "value": ws / (ms * 1e-3),
+                     "unit": "setups/s", "higher_is_better": True,
+                     "config": {"workload": CONFIGS["C5"][4], "block": b, "rows_per_gpu": n, "applies": napply},
+                     "breakdown_ms": {"setup": setup_ms, "apply": apply_ms},
+                     "step_hbm": {"algorithmic_bytes": ext_bytes + getrf_bytes + napply * getrs_bytes,
+                                  "achieved_gbs": (ext_bytes + getrf_bytes + napply * getrs_bytes) / (ms * 1e-3) / 1e9},
+                     "roofline": {"bound": "hbm", "kernel": "bj_apply", "achieved": getrs_bytes / (apply_ms * 1e-3) / 1e9,
+                                  "peak": hbm, "unit": "GB/s", "frac": getrs_bytes / (apply_ms * 1e-3) / 1e9 / hbm,
+                                  "traffic": None, "peak_source": peak_src, "bytes_per_launch": getrs_bytes}})
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -384,6 +482,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
     ap.add_argument("--nblocks", type=int, default=0, help="override blocks per GPU")
+    ap.add_argument("--block", type=int, default=0, help="C4/C5 diagonal block size (default 24)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
@@ -396,7 +495,10 @@ def main():
         run_reference(args, ws, rank)
         return
     ws, rank, local = dist_setup(args)
-    run_ours(args, ws, rank, local)
+    if args.config in FEM:
+        run_fem(args, ws, rank, local)
+    else:
+        run_ours(args, ws, rank, local)
     if ws > 1:
         dist.barrier()
         dist.destroy_process_group()
