@@ -96,12 +96,32 @@ constexpr int kFastShflW32 = 1, kFastPreRcp = 2;
 #define BJ_FAST_DEFAULT 0
 #endif
 
-template <typename R, int M, int F>
-__device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const int64_t *__restrict__ val_off,
+// Staging-buffer stride per tile: T*T elements rounded up to 16 bytes (the
+// bulk copy needs 16-B aligned destinations); 32/T tiles fit in 1024 elements.
+template <typename R>
+__host__ __device__ constexpr int stage_stride(int T) {
+    return (T * T + (16 / (int)sizeof(R)) - 1) / (16 / (int)sizeof(R)) * (16 / (int)sizeof(R));
+}
+
+// Per-lane view of one task (G = 32 / T blocks of one order): the lane's
+// tile's block id and global position.  Fetched two tasks ahead.
+struct FTask {
+    int m;            // order (warp-uniform), 0 = no task
+    bool ok;          // this lane's tile has a block
+    int blk;
+    int64_t lo;       // val_off[blk]
+    int64_t vo;       // vec_off[blk]
+};
+
+// S: this tile's block staged in shared memory by the bulk copy (column-major,
+// leading dimension M); `after_load` runs once the block is in registers
+// (it re-arms the warp's staging buffer with the next task).
+template <typename R, int M, int F, class AfterLoad>
+__device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &tk, const R *S,
                                                 const int64_t *__restrict__ vec_off, int32_t *__restrict__ piv,
-                                                int32_t *__restrict__ info, const int32_t *__restrict__ order,
-                                                int64_t first, int64_t last, int32_t *__restrict__ safe_list,
-                                                unsigned *__restrict__ safe_count, FastSmem<R> &sm) {
+                                                int32_t *__restrict__ info, int32_t *__restrict__ safe_list,
+                                                unsigned *__restrict__ safe_count, FastSmem<R> &sm,
+                                                AfterLoad &&after_load) {
     constexpr int T = tile_width(M);
     constexpr bool W32 = (T == 32) && ((F & kFastShflW32) != 0);
     constexpr bool PRE = (F & kFastPreRcp) != 0;
@@ -109,18 +129,18 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const int64_t
     const int t = lane / T;
     const int r = lane % T;
     const int tbase = t * T;
-    const int64_t idx = first + t;
-    bool tile_ok = idx < last;
-    const int blk = tile_ok ? __ldg(order + idx) : 0;
-    R *Ab = A + (tile_ok ? __ldg(val_off + blk) : 0);
+    bool tile_ok = tk.ok;
+    const int blk = tk.blk;
+    R *Ab = A + tk.lo;
 
     R a[M];
     bool ok = true;
     static_for<0, M>([&](auto jc) {
         constexpr int j = decltype(jc)::value;
-        a[j] = (tile_ok && r < M) ? Ab[r + j * M] : R(0);
+        a[j] = (tile_ok && r < M) ? S[r + j * M] : R(0);
         ok = ok && zero_mult_safe(a[j]);
     });
+    after_load();
     // Tiles with an entry outside the fast path's precondition go to the safe kernel.
     if (tile_bits<T>(__ballot_sync(kFull, !ok), tbase) != 0u) {
         if (tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
@@ -247,29 +267,75 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const int64_t
             constexpr int j = decltype(jc)::value;
             Ab[pos + j * M] = a[j];
         });
-        piv[__ldg(vec_off + blk) + pos] = r;
+        piv[tk.vo + pos] = r;
     }
     if (tile_ok && r == 0) info[blk] = inf;
 }
 
-template <typename R, int M, int MHI, int F>
-__device__ __forceinline__ void getrf_fast_dispatch(int m, R *A, const int64_t *val_off, const int64_t *vec_off,
-                                                    int32_t *piv, int32_t *info, const int32_t *order,
-                                                    int64_t first, int64_t last, int32_t *safe_list,
-                                                    unsigned *safe_count, FastSmem<R> &sm) {
-    if (m == M) {
-        getrf_fast_tile<R, M, F>(A, val_off, vec_off, piv, info, order, first, last, safe_list, safe_count, sm);
+template <typename R, int M, int MHI, int F, class AfterLoad>
+__device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const R *S, const int64_t *vec_off,
+                                                    int32_t *piv, int32_t *info, int32_t *safe_list,
+                                                    unsigned *safe_count, FastSmem<R> &sm, AfterLoad &&after_load) {
+    if (tk.m == M) {
+        constexpr int T = tile_width(M);
+        getrf_fast_tile<R, M, F>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), vec_off, piv, info,
+                                 safe_list, safe_count, sm, after_load);
     } else {
         if constexpr (M < MHI)
-            getrf_fast_dispatch<R, M + 1, MHI, F>(m, A, val_off, vec_off, piv, info, order, first, last, safe_list,
-                                               safe_count, sm);
+            getrf_fast_dispatch<R, M + 1, MHI, F>(A, tk, S, vec_off, piv, info, safe_list, safe_count, sm,
+                                                  after_load);
     }
 }
 
+template <int NM>
+__device__ __forceinline__ FTask getrf_fetch(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
+                                             const int64_t *s_first, const int64_t *s_last,
+                                             const int32_t *__restrict__ order, const int64_t *__restrict__ val_off,
+                                             const int64_t *__restrict__ vec_off) {
+    FTask tk;
+    tk.m = 0;
+    tk.ok = false;
+    tk.blk = 0;
+    tk.lo = 0;
+    tk.vo = 0;
+    if (task >= ntask) return tk;
+    int i = 0;
+    while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
+    const int m = mlo + i;
+    const int64_t idx = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m) + (threadIdx.x & 31) / tile_width(m);
+    tk.m = m;
+    tk.ok = idx < s_last[i];
+    tk.blk = tk.ok ? __ldg(order + idx) : 0;
+    tk.lo = tk.ok ? __ldg(val_off + tk.blk) : 0;
+    tk.vo = tk.ok ? __ldg(vec_off + tk.blk) : 0;
+    return tk;
+}
+
+// Stage task tk's blocks into the warp's buffer S: tile t's block (m*m
+// elements, rounded up to 16 B -- the rounding stays inside the block's
+// 16-B aligned slot) goes to S + t*stage_stride(T).  Lane 0 posts the byte count, then
+// each tile's lane 0 issues one bulk copy.
+template <typename R>
+__device__ __forceinline__ void getrf_stage(R *A, const FTask &tk, R *S, uint64_t *bar) {
+    if (tk.m == 0) return;
+    const int lane = threadIdx.x & 31;
+    const int T = tile_width(tk.m);
+    const unsigned bytes = (unsigned)((tk.m * tk.m * (int)sizeof(R) + 15) & ~15);
+    const unsigned lead = __ballot_sync(kFull, tk.ok && (lane % T) == 0);
+    if (lane == 0) mbar_expect_tx(bar, bytes * __popc(lead));
+    __syncwarp();
+    if (tk.ok && (lane % T) == 0) bulk_g2s(S + (lane / T) * stage_stride<R>(T), A + tk.lo, bytes, bar);
+}
+
 // One size class [MLO, MHI].  Tasks enumerated bin by bin; warp w takes tasks
-// w, w + nwarps, ...
+// w, w + nwarps, ...  Each warp owns an 8-KB staging buffer: while it factors
+// task i from registers, the bulk copy of task i+1 is in flight (and task
+// i+2's indices), so the block load no longer waits on HBM latency.
+#ifndef BJ_FAST_MINB
+#define BJ_FAST_MINB(R) (sizeof(R) == 8 ? 3 : 4)   // scripts/micro/getrf_bench.cu (B200): fp64 12 warps/SM beat 16, 20; fp32 16
+#endif
 template <typename R, int MLO, int MHI, int F = BJ_FAST_DEFAULT>
-__global__ void __launch_bounds__(kFastThreads, 4)
+__global__ void __launch_bounds__(kFastThreads, BJ_FAST_MINB(R))
 k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off,
              int32_t *__restrict__ piv, int32_t *__restrict__ info, const int32_t *__restrict__ order,
              const int64_t *__restrict__ bin_start, int32_t *__restrict__ safe_list,
@@ -277,6 +343,9 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     constexpr int NM = MHI - MLO + 1;
     __shared__ int64_t s_pref[NM + 1], s_first[NM], s_last[NM];
     __shared__ __align__(16) FastSmem<R> s_warp[kFastThreads / 32];
+    __shared__ __align__(128) R s_stage[kFastThreads / 32][32 * 32];
+    __shared__ __align__(8) uint64_t s_bar[kFastThreads / 32];
+    const int w = threadIdx.x >> 5;
     if (threadIdx.x == 0) {
         int64_t acc = 0;
         for (int i = 0; i < NM; ++i) {
@@ -290,17 +359,33 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
         }
         s_pref[NM] = acc;
     }
+    if ((threadIdx.x & 31) == 0) mbar_init(&s_bar[w], 1);
     __syncthreads();
     const int64_t ntask = s_pref[NM];
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    FastSmem<R> &sm = s_warp[threadIdx.x >> 5];
-    for (int64_t task = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; task < ntask; task += nwarps) {
-        int i = 0;
-        while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
-        const int m = MLO + i;
-        const int64_t first = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m);
-        getrf_fast_dispatch<R, MLO, MHI, F>(m, A, val_off, vec_off, piv, info, order, first, s_last[i], safe_list,
-                                         safe_count, sm);
+    FastSmem<R> &sm = s_warp[w];
+    R *S = s_stage[w];
+    uint64_t *bar = &s_bar[w];
+    // Warp index through a warp reduction: the compiler then treats task and
+    // order m as warp-uniform and emits plain SHFL/REDUX/VOTE in the
+    // size-specialised code instead of collective-emulation sequences.
+    const int64_t warp = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5));
+    FTask cur = getrf_fetch<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
+    FTask nxt = getrf_fetch<NM>(warp + nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
+    getrf_stage(A, cur, S, bar);
+    unsigned parity = 0;
+    for (int64_t task = warp; task < ntask; task += nwarps) {
+        const FTask nn = getrf_fetch<NM>(task + 2 * nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
+        mbar_wait_warp(bar, parity);
+        parity ^= 1u;
+        auto after_load = [&]() {
+            __syncwarp();                 // every lane has its block in registers
+            fence_proxy_async_smem();
+            getrf_stage(A, nxt, S, bar);
+        };
+        getrf_fast_dispatch<R, MLO, MHI, F>(A, cur, S, vec_off, piv, info, safe_list, safe_count, sm, after_load);
+        cur = nxt;
+        nxt = nn;
     }
 }
 
@@ -310,6 +395,7 @@ bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off
     static int grid = 0;
     if (grid == 0) {
         int per_sm = 0;
+        cudaFuncSetAttribute(k_getrf_fast<R, MLO, MHI>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrf_fast<R, MLO, MHI>, kFastThreads, 0);
         grid = (per_sm < 1 ? 1 : per_sm) * sm_count();
     }

@@ -2,13 +2,11 @@
 // getrs_kernels.cuh -- hot-path rows a4/a5: batched GETRS, P:218-238 steps 2-4,
 // section III.B, Fig. 2 bottom (eager, column-oriented).
 //
-// Same size-class / tile structure as getrf.cu.  Lane r of a tile holds row r
-// of L\U (read column by column: coalesced) and one element of the
-// right-hand side, loaded through the permutation (b := P b while
-// distributing b over the lanes).  The eager lower solve
-// broadcasts y_k and every lane below applies one fused AXPY term; the upper
-// solve (mirrored, R8) divides y_k by U(k,k) in lane k first.  Every y_i
-// receives the same sequence of correctly rounded operations as the oracle.
+// Same size classes as getrf.cu; the tile (getrs_tile.cuh) gives each lane
+// up to 4 rows and each warp 32 / rs_lanes(m) blocks.  The eager lower solve
+// broadcasts y_k and every row below applies one fused AXPY term; the upper
+// solve (mirrored, R8) divides y_k by U(k,k) first.  Every y_i receives the
+// same sequence of correctly rounded operations as the oracle.
 #include "common.cuh"
 #include "internal.h"
 #include "getrs_tile.cuh"
@@ -16,27 +14,65 @@
 namespace bj {
 
 constexpr int kGetrsThreads = 128;
+#ifndef BJ_RS_DEPTH
+#define BJ_RS_DEPTH 4   // scripts/micro/getrs_bench.cu sweep (B200): 4 ~ 12 > 8 > 16
+#endif
+#ifndef BJ_RS_MINB
+#define BJ_RS_MINB 4
+#endif
+
+// Per-lane metadata of one task (G blocks), loaded one task ahead so the
+// dependent index chain order -> offsets -> perm overlaps the previous solve.
+struct RsTask {
+    int m;                 // block order (warp-uniform), 0 = no task
+    bool ok;               // this lane's tile has a block
+    int64_t vo, lo;        // vec_off / val_off of the tile's block
+    int pv[4];             // perm of the lane's rows (q + s T)
+};
+
+template <int NM>
+__device__ __forceinline__ RsTask rs_fetch(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
+                                           const int64_t *s_first, const int64_t *s_last, const int32_t *order,
+                                           const int64_t *val_off, const int64_t *vec_off, const int32_t *piv) {
+    RsTask t;
+    t.m = 0;
+    t.ok = false;
+    t.vo = t.lo = 0;
+    t.pv[0] = t.pv[1] = t.pv[2] = t.pv[3] = 0;
+    if (task >= ntask) return t;
+    int i = 0;
+    while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
+    const int m = mlo + i;
+    const int T = rs_lanes(m);
+    const int lane = threadIdx.x & 31;
+    const int64_t last = s_last[i];
+    const int64_t idx = s_first[i] + (task - s_pref[i]) * rs_tiles(m) + lane / T;
+    t.m = m;
+    t.ok = idx < last;
+    const int blk = __ldg(order + (t.ok ? idx : last - 1));   // clamped: see getrs_rows
+    t.vo = __ldg(vec_off + blk);
+    t.lo = __ldg(val_off + blk);
+    const int q = lane % T;
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+        const int r = q + s * T;
+        t.pv[s] = r < m ? __ldg(piv + t.vo + r) : 0;
+    }
+    return t;
+}
 
 template <typename R, int M, int MHI>
-__device__ __forceinline__ void getrs_dispatch(int m, const R *LU, const int64_t *val_off, const int64_t *vec_off,
-                                               const int32_t *piv, const R *b, R *x, const int32_t *order,
-                                               int64_t first, int64_t last) {
-    if (m == M) {
-        const int lane = threadIdx.x & 31;
-        constexpr int T = tile_width(M);
-        const int64_t idx = first + lane / T;
-        const bool tile_ok = idx < last;
-        const int blk = tile_ok ? __ldg(order + idx) : 0;
-        const int64_t vo = tile_ok ? __ldg(vec_off + blk) : 0;
-        const int64_t lo = tile_ok ? __ldg(val_off + blk) : 0;
-        getrs_tile<R, M>(LU + lo, piv + vo, b + vo, x + vo, tile_ok);
+__device__ __forceinline__ void getrs_dispatch(const RsTask &t, const R *LU, const int32_t *piv, const R *b, R *x) {
+    if (t.m == M) {
+        constexpr int T = rs_lanes(M);
+        getrs_rows<R, M, BJ_RS_DEPTH>(LU + t.lo, piv + t.vo, b + t.vo, x + t.vo, t.ok, (threadIdx.x & 31) % T, t.pv);
     } else {
-        if constexpr (M < MHI) getrs_dispatch<R, M + 1, MHI>(m, LU, val_off, vec_off, piv, b, x, order, first, last);
+        if constexpr (M < MHI) getrs_dispatch<R, M + 1, MHI>(t, LU, piv, b, x);
     }
 }
 
 template <typename R, int MLO, int MHI>
-__global__ void __launch_bounds__(kGetrsThreads)
+__global__ void __launch_bounds__(kGetrsThreads, BJ_RS_MINB)
 k_getrs_class(const R *__restrict__ LU, const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off,
               const int32_t *__restrict__ piv, const R *b, R *x, const int32_t *__restrict__ order,
               const int64_t *__restrict__ bin_start) {
@@ -47,7 +83,7 @@ k_getrs_class(const R *__restrict__ LU, const int64_t *__restrict__ val_off, con
         for (int i = 0; i < NM; ++i) {
             const int m = MLO + i;
             const int64_t b0 = bin_start[m], b1 = bin_start[m + 1];
-            const int g = tiles_per_warp(m);
+            const int g = rs_tiles(m);
             s_first[i] = b0;
             s_last[i] = b1;
             s_pref[i] = acc;
@@ -58,12 +94,17 @@ k_getrs_class(const R *__restrict__ LU, const int64_t *__restrict__ val_off, con
     __syncthreads();
     const int64_t ntask = s_pref[NM];
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t task = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; task < ntask; task += nwarps) {
-        int i = 0;
-        while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
-        const int m = MLO + i;
-        const int64_t first = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m);
-        getrs_dispatch<R, MLO, MHI>(m, LU, val_off, vec_off, piv, b, x, order, first, s_last[i]);
+    // The warp index goes through a warp reduction so the compiler sees it
+    // (and everything derived from it: task, order m) as warp-uniform; the
+    // shuffles inside the size-specialised code are then plain SHFLs rather
+    // than collective-emulation sequences.
+    const int64_t warp = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5));
+    RsTask cur = rs_fetch<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off, piv);
+    for (int64_t task = warp; task < ntask; task += nwarps) {
+        const RsTask nxt = rs_fetch<NM>(task + nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off,
+                                        piv);
+        getrs_dispatch<R, MLO, MHI>(cur, LU, piv, b, x);
+        cur = nxt;
     }
 }
 

@@ -6,7 +6,7 @@
 #include <vector>
 #include <algorithm>
 #include "getrf_kernels.cuh"
-#include "getrf_fast.cuh"
+#include "getrf_r2_experiment.cuh"
 
 namespace bj {
 void count_launch(int) {}
@@ -188,22 +188,76 @@ void run(int64_t nb, const char *name, int force_warps_per_sm = 0) {
     cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
 }
 
-int main() {
+template <typename R>
+void run_r2(int64_t nb, int LO, int HI, const char *name) {
+    std::vector<int64_t> vo(nb + 1), ve(nb + 1);
+    std::vector<int32_t> ord(nb);
+    std::vector<int64_t> cnt(kBins + 1, 0);
+    std::vector<int> m_of(nb);
+    const int el = 16 / (int)sizeof(R);
+    for (int64_t i = 0; i < nb; ++i) m_of[i] = LO + (int)((i * (HI - LO + 1)) / nb);
+    vo[0] = 0; ve[0] = 0;
+    for (int64_t i = 0; i < nb; ++i) { int m = m_of[i]; vo[i + 1] = vo[i] + (m * m + el - 1) / el * el; ve[i + 1] = ve[i] + m; ord[i] = (int32_t)i; cnt[m]++; }
+    std::vector<int64_t> bs(kBins + 1, 0);
+    int64_t acc = 0;
+    for (int b = 0; b < kBins; ++b) { bs[b] = acc; acc += cnt[b]; }
+    bs[kBins] = acc;
+    R *A, *A0; int64_t *dvo, *dve, *dbs; int32_t *dord, *piv, *info, *list; unsigned *count;
+    const int64_t tot = vo[nb];
+    cudaMalloc(&A, tot * sizeof(R)); cudaMalloc(&A0, tot * sizeof(R));
+    cudaMalloc(&dvo, (nb + 1) * 8); cudaMalloc(&dve, (nb + 1) * 8); cudaMalloc(&dbs, (kBins + 1) * 8);
+    cudaMalloc(&dord, nb * 4); cudaMalloc(&piv, ve[nb] * 4); cudaMalloc(&info, nb * 4); cudaMalloc(&list, nb * 4);
+    cudaMalloc(&count, 4);
+    cudaMemcpy(dvo, vo.data(), (nb + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dve, ve.data(), (nb + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dbs, bs.data(), (kBins + 1) * 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(dord, ord.data(), nb * 4, cudaMemcpyHostToDevice);
+    {
+        std::vector<R> h(tot);
+        unsigned long long z = 88172645463325252ull;
+        for (int64_t i = 0; i < tot; ++i) { z ^= z << 13; z ^= z >> 7; z ^= z << 17; h[i] = (R)((double)(z >> 11) * 0x1p-52 - 1.0); }
+        cudaMemcpy(A0, h.data(), tot * sizeof(R), cudaMemcpyHostToDevice);
+    }
+    PlanView pv; pv.nblocks = nb; pv.order = dord; pv.bin_start = dbs;
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    std::vector<float> ts;
+    unsigned hc = 0;
+    for (int rep = 0; rep < 6; ++rep) {
+        cudaMemcpy(A, A0, tot * sizeof(R), cudaMemcpyDeviceToDevice);
+        cudaMemset(count, 0, 4);
+        cudaEventRecord(e0);
+        launch_getrf_r2<R>(A, dvo, dve, piv, info, pv, list, count, 0);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        if (rep) ts.push_back(ms);
+        cudaMemcpy(&hc, count, 4, cudaMemcpyDeviceToHost);
+    }
+    std::sort(ts.begin(), ts.end());
+    double bytes = 0;
+    for (int64_t i = 0; i < nb; ++i) bytes += 2.0 * sizeof(R) * m_of[i] * m_of[i] + 4 * m_of[i] + 20;
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrf_r2<R>, kR2Threads, r2_dyn_smem(sizeof(R)));
+    printf("R2 sel=%d minb=%d %-22s occ=%d warps/SM  %8.1f us  %7.1f GB/s  %6.1f Mblk/s  deferred=%u err=%s\n",
+           BJ_R2_SELECT, BJ_R2_MINB, name, per_sm * 4, ts[ts.size() / 2] * 1e3, bytes / (ts[ts.size() / 2] * 1e-3) / 1e9,
+           nb / (ts[ts.size() / 2] * 1e-3) / 1e6, hc, cudaGetErrorString(cudaGetLastError()));
+    cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
+    cudaFree(list); cudaFree(count);
+}
+
+int main(int argc, char **argv) {
 #ifdef BJ_TRACE
     run_fast1<32>(148, "FAST 1 warp");
-    run_fast1<24>(148, "FAST 1 warp");
-    run_fast1<16>(296, "FAST 1 warp");
 #else
-    run_mix<17, 32, 0>(552000, "mix smem base (old)");
+    if (argc > 1) {
+        run_r2<double>(40000, 32, 32, "m=32 f64");
+        run_r2<double>(552000, 17, 32, "mix 17..32 f64");
+        run_r2<float>(552000, 17, 32, "mix 17..32 f32");
+        return 0;
+    }
+    run_mix_fast<32, 32, 0>(40000, "m=32 F0 smem");
     run_mix_fast<17, 32, 0>(552000, "mix FAST F0 smem");
-    run_mix_fast<17, 32, 1>(552000, "mix FAST F1 shfl");
-    run_mix_fast<17, 32, 2>(552000, "mix FAST F2 smem+pre");
-    run_mix<9, 16, 0>(276000, "mix9-16 old");
     run_mix_fast<9, 16, 0>(276000, "mix9-16 FAST F0");
-    run_mix_fast<9, 16, 2>(276000, "mix9-16 FAST F2");
-    run_mix<5, 8, 0>(138000, "mix5-8 old");
-    run_mix_fast<5, 8, 0>(138000, "mix5-8 FAST F0");
-    run_mix_fast<1, 4, 0>(69000, "mix1-4 FAST F0");
 #endif
     return 0;
 }
