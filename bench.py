@@ -263,7 +263,7 @@ def run_ours(args, ws, rank, local):
     # warm-up
     keep = []
     for i in range(args.warmup):
-        keep.append(one_step(pool[i % pool_n]))
+        one_step(pool[i % pool_n]).close()     # stream-ordered free, no sync
     barrier(ws)
     for p in keep:
         p.close()
@@ -289,7 +289,7 @@ def run_ours(args, ws, rank, local):
             bj.launch_count_reset()
             start.record(stream)
             for i in range(n):
-                keep.append(one_step(pool[i], evs[i]))
+                one_step(pool[i], evs[i]).close()
             end.record(stream)
             launches += bj.launch_count()
             barrier(ws)

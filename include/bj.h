@@ -111,6 +111,9 @@ bj_status bj_layout_from_block_ptr(int64_t nblocks, const int32_t *block_ptr, bj
  * wants to reuse it (the plan copies what it needs). */
 bj_status bj_plan_create(bj_plan **plan, int64_t nblocks, const int32_t *sizes,
                          bj_stream_t stream);
+/* Frees the plan's device memory stream-ordered on the creation stream (no
+ * host sync): work already enqueued on that stream may still use it; work on
+ * other streams must be ordered before this call by the caller. */
 bj_status bj_plan_destroy(bj_plan *plan);
 
 /* ---------------------------------------------------------------------------

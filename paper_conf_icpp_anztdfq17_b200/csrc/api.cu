@@ -45,6 +45,7 @@ struct bj_plan {
     int64_t nblocks = 0;
     int32_t *order = nullptr;
     int64_t *bin_start = nullptr;
+    cudaStream_t stream = nullptr;     // creation stream: the plan's memory is freed on it
     PlanView view() const { return PlanView{nblocks, order, bin_start}; }
 };
 
@@ -61,8 +62,25 @@ struct bj_workspace {
     size_t cap = 0;
 };
 
+// The library's scratch and plan memory comes from the device's default
+// stream-ordered pool; keep freed memory in the pool (no release at stream
+// syncs) so per-call allocations never reach the driver on the hot path.
+static void pool_keep_memory() {
+    static bool done = false;
+    if (done) return;
+    done = true;
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t keep = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+}
+
 static bj_status plan_alloc_build(bj_plan *p, int64_t nb, const int32_t *sizes, cudaStream_t s) {
+    pool_keep_memory();
     p->nblocks = nb;
+    p->stream = s;
     BJ_CUDA_TRY(cudaMallocAsync((void **)&p->order, sizeof(int32_t) * (size_t)(nb > 0 ? nb : 1), s));
     BJ_CUDA_TRY(cudaMallocAsync((void **)&p->bin_start, sizeof(int64_t) * (kBins + 1), s));
     return build_plan(nb, sizes, p->order, p->bin_start, s);
@@ -125,8 +143,8 @@ bj_status bj_plan_create(bj_plan **plan, int64_t nblocks, const int32_t *sizes, 
 
 bj_status bj_plan_destroy(bj_plan *plan) {
     if (!plan) return BJ_ERR_ARG;
-    if (plan->order) cudaFree(plan->order);
-    if (plan->bin_start) cudaFree(plan->bin_start);
+    // stream-ordered: after every call already enqueued on the creation stream
+    plan_free_async(plan, plan->stream);
     delete plan;
     return BJ_OK;
 }

@@ -91,7 +91,7 @@ struct FastSmem {
 // C3 order mix): kFastShflW32 -- full-warp tiles broadcast by SHFL instead of
 // smem; kFastPreRcp -- every lane pre-refines 1/a_kk (shorter chain, more
 // instructions).
-constexpr int kFastShflW32 = 1, kFastPreRcp = 2;
+constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4;
 #ifndef BJ_FAST_DEFAULT
 #define BJ_FAST_DEFAULT 0
 #endif
@@ -125,6 +125,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     constexpr int T = tile_width(M);
     constexpr bool W32 = (T == 32) && ((F & kFastShflW32) != 0);
     constexpr bool PRE = (F & kFastPreRcp) != 0;
+    constexpr bool HYB = (T == 32) && !W32 && ((F & kFastHybrid) != 0);
     const int lane = threadIdx.x & 31;
     const int t = lane / T;
     const int r = lane % T;
@@ -162,7 +163,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         R y = R(0);
         if constexpr (PRE) {
             y = Num<R>::rcp_refine(a[k]);
-            if constexpr (!W32) {
+            if constexpr (!W32 && !HYB) {
                 if constexpr (sizeof(R) == 8) *reinterpret_cast<double2 *>(sm.slot + 2 * lane) = make_double2(a[k], y);
                 else *reinterpret_cast<float2 *>(sm.slot + 2 * lane) = make_float2(a[k], y);
             }
@@ -179,8 +180,25 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         // line 12: the pivot (and its reciprocal)
         const bool isp = (r == ipiv) && row_ok;
         if (isp) tag = k + 1;                                   // line 9
-        R d, yd;
-        if constexpr (W32) {
+        R d, yd, u1 = R(0);
+        if constexpr (HYB) {
+            // critical-path values straight from the pivot lane (warp-uniform
+            // source), issued before the row publish; the rest of the pivot
+            // row (columns >= k+2) goes through shared memory.
+            d = __shfl_sync(kFull, a[k], ipiv);
+            if constexpr (k + 1 < M) u1 = __shfl_sync(kFull, a[k + 1], ipiv);
+            if constexpr (PRE) yd = __shfl_sync(kFull, y, ipiv);
+            else yd = Num<R>::rcp_refine(d);
+            if constexpr (k + 2 < M) {
+                constexpr int j0 = (k + 2) & ~1;
+                static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
+                    constexpr int j = j0 + 2 * decltype(pc)::value;
+                    if constexpr (j + 1 < M) st_shared_pred(isp, buf + j, a[j], a[j + 1]);
+                    else st_shared_pred(isp, buf + j, a[j]);
+                });
+            }
+            __syncwarp();
+        } else if constexpr (W32) {
             d = __shfl_sync(kFull, a[k], ipiv);
             if constexpr (PRE) yd = __shfl_sync(kFull, y, ipiv);
             else yd = Num<R>::rcp_refine(d);
@@ -225,7 +243,27 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         if (upd) a[k] = q;
         if (sing && inf == 0) inf = k + 1;
         // lines 14-15 (GER), branch-free
-        if constexpr (W32) {
+        if constexpr (HYB) {
+            if constexpr (k + 1 < M) a[k + 1] = Num<R>::fma(-l, u1, a[k + 1]);
+            if constexpr (((k + 2) & 1) && k + 2 < M) a[k + 2] = Num<R>::fma(-l, buf[k + 2], a[k + 2]);
+            constexpr int g0 = (k + 3) & ~1;
+            static_for<0, (g0 < M ? (M - g0 + 1) / 2 : 0)>([&](auto pc) {
+                constexpr int j = g0 + 2 * decltype(pc)::value;
+                if constexpr (j + 1 < M) {
+                    if constexpr (sizeof(R) == 8) {
+                        const double2 u = *reinterpret_cast<const double2 *>(buf + j);
+                        a[j] = Num<R>::fma(-l, u.x, a[j]);
+                        a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
+                    } else {
+                        const float2 u = *reinterpret_cast<const float2 *>(buf + j);
+                        a[j] = Num<R>::fma(-l, u.x, a[j]);
+                        a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
+                    }
+                } else {
+                    a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                }
+            });
+        } else if constexpr (W32) {
             static_for<k + 1, M>([&](auto jc) {
                 constexpr int j = decltype(jc)::value;
                 const R u = __shfl_sync(kFull, a[j], ipiv);
@@ -287,11 +325,14 @@ __device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const
     }
 }
 
+// Task indices in two stages so no load waits on the one before it inside
+// an iteration: getrf_fetch_idx (order[]) runs three tasks ahead,
+// getrf_fetch_off (val_off/vec_off of the block found one iteration earlier)
+// two tasks ahead.
 template <int NM>
-__device__ __forceinline__ FTask getrf_fetch(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
-                                             const int64_t *s_first, const int64_t *s_last,
-                                             const int32_t *__restrict__ order, const int64_t *__restrict__ val_off,
-                                             const int64_t *__restrict__ vec_off) {
+__device__ __forceinline__ FTask getrf_fetch_idx(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
+                                                 const int64_t *s_first, const int64_t *s_last,
+                                                 const int32_t *__restrict__ order) {
     FTask tk;
     tk.m = 0;
     tk.ok = false;
@@ -306,9 +347,12 @@ __device__ __forceinline__ FTask getrf_fetch(int64_t task, int64_t ntask, int ml
     tk.m = m;
     tk.ok = idx < s_last[i];
     tk.blk = tk.ok ? __ldg(order + idx) : 0;
+    return tk;
+}
+__device__ __forceinline__ void getrf_fetch_off(FTask &tk, const int64_t *__restrict__ val_off,
+                                                const int64_t *__restrict__ vec_off) {
     tk.lo = tk.ok ? __ldg(val_off + tk.blk) : 0;
     tk.vo = tk.ok ? __ldg(vec_off + tk.blk) : 0;
-    return tk;
 }
 
 // Stage task tk's blocks into the warp's buffer S: tile t's block (m*m
@@ -370,12 +414,16 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     // order m as warp-uniform and emits plain SHFL/REDUX/VOTE in the
     // size-specialised code instead of collective-emulation sequences.
     const int64_t warp = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5));
-    FTask cur = getrf_fetch<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
-    FTask nxt = getrf_fetch<NM>(warp + nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
+    FTask cur = getrf_fetch_idx<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order);
+    FTask nxt = getrf_fetch_idx<NM>(warp + nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+    FTask nn = getrf_fetch_idx<NM>(warp + 2 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+    getrf_fetch_off(cur, val_off, vec_off);
+    getrf_fetch_off(nxt, val_off, vec_off);
     getrf_stage(A, cur, S, bar);
     unsigned parity = 0;
     for (int64_t task = warp; task < ntask; task += nwarps) {
-        const FTask nn = getrf_fetch<NM>(task + 2 * nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off);
+        const FTask n3 = getrf_fetch_idx<NM>(task + 3 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+        getrf_fetch_off(nn, val_off, vec_off);
         mbar_wait_warp(bar, parity);
         parity ^= 1u;
         auto after_load = [&]() {
@@ -386,6 +434,7 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
         getrf_fast_dispatch<R, MLO, MHI, F>(A, cur, S, vec_off, piv, info, safe_list, safe_count, sm, after_load);
         cur = nxt;
         nxt = nn;
+        nn = n3;
     }
 }
 

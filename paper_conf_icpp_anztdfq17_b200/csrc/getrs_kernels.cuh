@@ -15,28 +15,32 @@ namespace bj {
 
 constexpr int kGetrsThreads = 128;
 #ifndef BJ_RS_DEPTH
-#define BJ_RS_DEPTH 4   // scripts/micro/getrs_bench.cu sweep (B200): 4 ~ 12 > 8 > 16
+#define BJ_RS_DEPTH 12   // scripts/micro/getrs_bench.cu sweep (B200, 3-stage index pipeline): 12 > 4
 #endif
 #ifndef BJ_RS_MINB
 #define BJ_RS_MINB 4
 #endif
 
-// Per-lane metadata of one task (G blocks), loaded one task ahead so the
-// dependent index chain order -> offsets -> perm overlaps the previous solve.
+// Per-lane metadata of one task (G blocks).  The dependent index chain
+// order -> offsets -> perm is pipelined across iterations: rs_fetch_idx runs
+// three tasks ahead, rs_fetch_off two, rs_fetch_piv one, so no load waits on
+// another inside an iteration.
 struct RsTask {
     int m;                 // block order (warp-uniform), 0 = no task
     bool ok;               // this lane's tile has a block
+    int blk;
     int64_t vo, lo;        // vec_off / val_off of the tile's block
     int pv[4];             // perm of the lane's rows (q + s T)
 };
 
 template <int NM>
-__device__ __forceinline__ RsTask rs_fetch(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
-                                           const int64_t *s_first, const int64_t *s_last, const int32_t *order,
-                                           const int64_t *val_off, const int64_t *vec_off, const int32_t *piv) {
+__device__ __forceinline__ RsTask rs_fetch_idx(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
+                                               const int64_t *s_first, const int64_t *s_last,
+                                               const int32_t *order) {
     RsTask t;
     t.m = 0;
     t.ok = false;
+    t.blk = 0;
     t.vo = t.lo = 0;
     t.pv[0] = t.pv[1] = t.pv[2] = t.pv[3] = 0;
     if (task >= ntask) return t;
@@ -49,16 +53,23 @@ __device__ __forceinline__ RsTask rs_fetch(int64_t task, int64_t ntask, int mlo,
     const int64_t idx = s_first[i] + (task - s_pref[i]) * rs_tiles(m) + lane / T;
     t.m = m;
     t.ok = idx < last;
-    const int blk = __ldg(order + (t.ok ? idx : last - 1));   // clamped: see getrs_rows
-    t.vo = __ldg(vec_off + blk);
-    t.lo = __ldg(val_off + blk);
-    const int q = lane % T;
+    t.blk = __ldg(order + (t.ok ? idx : last - 1));   // clamped: see getrs_rows
+    return t;
+}
+__device__ __forceinline__ void rs_fetch_off(RsTask &t, const int64_t *val_off, const int64_t *vec_off) {
+    if (t.m == 0) return;
+    t.vo = __ldg(vec_off + t.blk);
+    t.lo = __ldg(val_off + t.blk);
+}
+__device__ __forceinline__ void rs_fetch_piv(RsTask &t, const int32_t *piv) {
+    if (t.m == 0) return;
+    const int T = rs_lanes(t.m);
+    const int q = (threadIdx.x & 31) % T;
 #pragma unroll
     for (int s = 0; s < 4; ++s) {
         const int r = q + s * T;
-        t.pv[s] = r < m ? __ldg(piv + t.vo + r) : 0;
+        t.pv[s] = r < t.m ? __ldg(piv + t.vo + r) : 0;
     }
-    return t;
 }
 
 template <typename R, int M, int MHI>
@@ -99,12 +110,20 @@ k_getrs_class(const R *__restrict__ LU, const int64_t *__restrict__ val_off, con
     // shuffles inside the size-specialised code are then plain SHFLs rather
     // than collective-emulation sequences.
     const int64_t warp = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5));
-    RsTask cur = rs_fetch<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off, piv);
+    RsTask cur = rs_fetch_idx<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order);
+    RsTask nxt = rs_fetch_idx<NM>(warp + nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+    RsTask nn = rs_fetch_idx<NM>(warp + 2 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+    rs_fetch_off(cur, val_off, vec_off);
+    rs_fetch_off(nxt, val_off, vec_off);
+    rs_fetch_piv(cur, piv);
     for (int64_t task = warp; task < ntask; task += nwarps) {
-        const RsTask nxt = rs_fetch<NM>(task + nwarps, ntask, MLO, s_pref, s_first, s_last, order, val_off, vec_off,
-                                        piv);
+        const RsTask n3 = rs_fetch_idx<NM>(task + 3 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
+        rs_fetch_off(nn, val_off, vec_off);
+        rs_fetch_piv(nxt, piv);
         getrs_dispatch<R, MLO, MHI>(cur, LU, piv, b, x);
         cur = nxt;
+        nxt = nn;
+        nn = n3;
     }
 }
 

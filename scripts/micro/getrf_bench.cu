@@ -256,8 +256,11 @@ int main(int argc, char **argv) {
         return 0;
     }
     run_mix_fast<32, 32, 0>(40000, "m=32 F0 smem");
+    run_mix_fast<32, 32, 4>(40000, "m=32 F4 hybrid");
+    run_mix_fast<32, 32, 6>(40000, "m=32 F6 hybrid+pre");
     run_mix_fast<17, 32, 0>(552000, "mix FAST F0 smem");
-    run_mix_fast<9, 16, 0>(276000, "mix9-16 FAST F0");
+    run_mix_fast<17, 32, 4>(552000, "mix FAST F4 hybrid");
+    run_mix_fast<17, 32, 6>(552000, "mix FAST F6 hybrid+pre");
 #endif
     return 0;
 }
