@@ -115,6 +115,7 @@ void bj_launch_count_reset(void) { g_launches = 0; }
 
 bj_status bj_layout(int64_t nblocks, const int32_t *sizes, bj_dtype dtype, int64_t *vec_off, int64_t *val_off,
                     bj_stream_t stream) {
+    pool_keep_memory();
     const int es = elem_size(dtype);
     if (nblocks < 0 || es == 0 || !vec_off || !val_off || (nblocks > 0 && !sizes)) return BJ_ERR_ARG;
     return layout_sizes(nblocks, sizes, es, vec_off, val_off, (cudaStream_t)stream);
@@ -122,6 +123,7 @@ bj_status bj_layout(int64_t nblocks, const int32_t *sizes, bj_dtype dtype, int64
 
 bj_status bj_layout_from_block_ptr(int64_t nblocks, const int32_t *block_ptr, bj_dtype dtype, int32_t *sizes,
                                    int64_t *vec_off, int64_t *val_off, bj_stream_t stream) {
+    pool_keep_memory();
     const int es = elem_size(dtype);
     if (nblocks < 0 || es == 0 || !block_ptr || !vec_off || !val_off || (nblocks > 0 && !sizes)) return BJ_ERR_ARG;
     return layout_block_ptr(nblocks, block_ptr, es, sizes, vec_off, val_off, (cudaStream_t)stream);
@@ -150,6 +152,7 @@ bj_status bj_plan_destroy(bj_plan *plan) {
 }
 
 bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out, bj_stream_t stream) {
+    pool_keep_memory();
     if (!A || !block_ptr) return BJ_ERR_ARG;
     bj_status st = check_batch(out, true);
     if (st != BJ_OK) return st;
@@ -163,6 +166,7 @@ bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out, b
 
 bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const bj_plan *plan,
                             bj_stream_t stream) {
+    pool_keep_memory();
     bj_status st = check_batch(blocks, true);
     if (st != BJ_OK) return st;
     if (blocks->nblocks > 0 && (!pivots || !info)) return BJ_ERR_ARG;
@@ -190,6 +194,7 @@ bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, co
 
 bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const void *b, void *x, const bj_plan *plan,
                             bj_stream_t stream) {
+    pool_keep_memory();
     bj_status st = check_batch(lu, true);
     if (st != BJ_OK) return st;
     if (lu->nblocks > 0 && (!pivots || !b || !x)) return BJ_ERR_ARG;
@@ -225,6 +230,7 @@ bj_status bj_create(bj_handle **handle) {
 
 bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *factors, int32_t *pivots,
                    int32_t *info, bj_stream_t stream) {
+    pool_keep_memory();
     if (!h || !A || !block_ptr || !factors) return BJ_ERR_ARG;
     bj_status st = check_batch(factors, true);
     if (st != BJ_OK) return st;
@@ -248,6 +254,7 @@ bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_b
 }
 
 bj_status bj_apply(bj_handle *h, const void *x, void *y, bj_stream_t stream) {
+    pool_keep_memory();
     if (!h || !x || !y) return BJ_ERR_ARG;
     if (!h->ready) return BJ_ERR_STATE;
     return bj_getrs_vbatched(&h->factors, h->pivots, x, y, &h->plan, stream);
@@ -300,6 +307,7 @@ static size_t up256(size_t x) { return (x + 255) & ~(size_t)255; }
 bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int64_t nvalues, const void *blocks_h,
                        int64_t nvec, const void *b_h, void *x_h, int32_t *pivots_h, int32_t *info_h, bj_dtype dtype,
                        bj_stream_t stream) {
+    pool_keep_memory();
     const int es = elem_size(dtype);
     if (!ws || nb < 0 || nvalues < 0 || nvec < 0 || es == 0) return BJ_ERR_ARG;
     if (nb > 0 && (!sizes_h || !blocks_h || !b_h || !x_h)) return BJ_ERR_ARG;

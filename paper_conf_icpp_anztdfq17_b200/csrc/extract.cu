@@ -16,6 +16,8 @@
 #include "common.cuh"
 #include "internal.h"
 
+#include <climits>
+
 namespace bj {
 
 constexpr int kExtractWarps = 4;
@@ -58,13 +60,39 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
         for (int i = lane; i < np; i += 32) T[i] = R(0);
         __syncwarp();
         const int64_t cb = (int64_t)bs + col_offset, ce = (int64_t)be + col_offset;
-        for (int r = 0; r < m; ++r) {
-            const int64_t rs = __shfl_sync(kFull, rpv, r);
-            const int64_t rn = __shfl_sync(kFull, rpv, (r + 1) & 31);
-            const int64_t re = r + 1 < m ? rn : e1;
-            for (int64_t e = rs + lane; e < re; e += 32) {
-                const int64_t c = __ldg(col_idx + e);
-                if (c >= cb && c < ce) T[r + (int)(c - cb) * m] = __ldg(values + e);
+        // The block's rows are one contiguous entry range [e0, e1): the warp
+        // scans it in 32-entry chunks (coalesced col-indices),
+        // kU chunks per round so kU loads per lane are in flight, and the
+        // value loads of one round overlap the col-index loads of the next.
+        // Row of entry e: rows starting at or before the chunk start (ballot)
+        // plus row starts inside the chunk at or before e (one REDUX.OR mask).
+        const int rel = lane < m ? (int)(rpv - e0) : INT_MAX;   // row start, relative
+        const int len = (int)(e1 - e0);
+        const int nch = (len + 31) >> 5;
+        constexpr int kU = 8;
+        int32_t cc[kU];
+        auto load_cols = [&](int c0) {
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int e = ((c0 + u) << 5) + lane;
+                cc[u] = e < len ? __ldg(col_idx + e0 + e) : -1;
+            }
+        };
+        load_cols(0);
+        for (int c0 = 0; c0 < nch; c0 += kU) {
+            int32_t cv[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) cv[u] = cc[u];
+            if (c0 + kU < nch) load_cols(c0 + kU);
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int E = (c0 + u) << 5;
+                if (E >= len) break;                                  // warp-uniform
+                const int row0 = __popc(__ballot_sync(kFull, rel <= E)) - 1;
+                const unsigned starts = __reduce_or_sync(kFull, (rel > E && rel < E + 32) ? 1u << (rel - E) : 0u);
+                const int row = row0 + __popc(starts & ((2u << lane) - 1u));
+                const int64_t c = cv[u];
+                if (c >= cb && c < ce) T[row + (int)(c - cb) * m] = __ldg(values + e0 + E + lane);
             }
         }
         __syncwarp();

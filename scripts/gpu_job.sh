@@ -1,10 +1,4 @@
-# round profiling job: tests, bench lines, ncu launch list + full-set summary
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.txt 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.txt
-python bench.py > gpurun_out/bench_C3.json 2>gpurun_out/bench_C3.err
-python bench.py --config C2 --steps 20 --warmup 3 --no-cpu > gpurun_out/bench_C2.json 2>gpurun_out/bench_C2.err
-python bench.py --config C3f32 --steps 20 --warmup 3 --no-cpu > gpurun_out/bench_C3f32.json 2>gpurun_out/bench_C3f32.err
-python bench.py --config C4 --steps 10 --warmup 3 --no-cpu > gpurun_out/bench_C4.json 2>gpurun_out/bench_C4.err
-python bench.py --config C5 --steps 5 --warmup 3 --no-cpu > gpurun_out/bench_C5.json 2>gpurun_out/bench_C5.err
-python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref.json 2>gpurun_out/bench_ref.err
-bash scripts/profile_round.sh C3 > gpurun_out/prof.log 2>&1
+python scripts/c4probe.py > gpurun_out/c4probe.txt 2>&1
+for b in 24 8 16 32; do python bench.py --config C4 --block $b --steps 10 --warmup 3 --no-e2e --no-cpu > gpurun_out/c4_$b.json 2>/dev/null; done
+python bench.py --steps 20 --warmup 3 --no-e2e --no-cpu > gpurun_out/c3.json 2>gpurun_out/c3.err
