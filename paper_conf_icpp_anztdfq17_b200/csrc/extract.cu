@@ -44,13 +44,35 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     R *T = tile[w];
     const int64_t nwarps = ((int64_t)gridDim.x * kExtractThreads) >> 5;
-    for (int64_t b = ((int64_t)blockIdx.x * kExtractThreads + threadIdx.x) >> 5; b < nb; b += nwarps) {
-        const int bs = __ldg(block_ptr + b), be = __ldg(block_ptr + b + 1);
+    // Block descriptors are pipelined across iterations: block_ptr two blocks
+    // ahead, row_ptr one block ahead, so a block's scan starts without
+    // waiting on its index chain.
+    const int64_t b0 = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * kExtractThreads + threadIdx.x) >> 5));
+    auto ld_bp = [&](int64_t b, int &bs, int &be) {
+        bs = b < nb ? __ldg(block_ptr + b) : 0;
+        be = b < nb ? __ldg(block_ptr + b + 1) : 0;
+    };
+    auto ld_rp = [&](int bs, int be, int64_t &rpv, int64_t &e1) {
+        const int m = be - bs;
+        rpv = (m > 0 && m <= kMaxM && lane < m) ? __ldg(row_ptr + bs + lane) : 0;
+        e1 = (m > 0 && m <= kMaxM) ? __ldg(row_ptr + be) : 0;
+    };
+    int n_bs, n_be, nn_bs, nn_be;
+    int64_t n_rpv, n_e1;
+    ld_bp(b0, n_bs, n_be);
+    ld_rp(n_bs, n_be, n_rpv, n_e1);
+    ld_bp(b0 + nwarps, nn_bs, nn_be);
+    for (int64_t b = b0; b < nb; b += nwarps) {
+        const int bs = n_bs, be = n_be;
+        const int64_t rpv = n_rpv, e1 = n_e1;
+        n_bs = nn_bs;
+        n_be = nn_be;
+        ld_rp(n_bs, n_be, n_rpv, n_e1);
+        ld_bp(b + 2 * nwarps, nn_bs, nn_be);
         const int m = be - bs;
         if (m <= 0 || m > kMaxM) continue;                     // nothing to write / invalid order
         // lane j < m holds row_ptr[bs + j]; every lane holds row_ptr[be]
-        const int64_t rpv = lane < m ? __ldg(row_ptr + bs + lane) : 0;
-        const int64_t e0 = __shfl_sync(kFull, rpv, 0), e1 = __ldg(row_ptr + be);
+        const int64_t e0 = __shfl_sync(kFull, rpv, 0);
         if (e1 - e0 > kHeavy) {
             if (lane == 0) heavy[atomicAdd(nheavy, 1ull)] = (int32_t)b;
             continue;
@@ -84,16 +106,30 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
 #pragma unroll
             for (int u = 0; u < kU; ++u) cv[u] = cc[u];
             if (c0 + kU < nch) load_cols(c0 + kU);
+            // all value loads of the round first (in-order issue: a store that
+            // waits on its load would otherwise serialise the chunks), then
+            // the scatter into the smem tile
+            R vv[kU];
+            int at[kU];
 #pragma unroll
             for (int u = 0; u < kU; ++u) {
                 const int E = (c0 + u) << 5;
-                if (E >= len) break;                                  // warp-uniform
-                const int row0 = __popc(__ballot_sync(kFull, rel <= E)) - 1;
-                const unsigned starts = __reduce_or_sync(kFull, (rel > E && rel < E + 32) ? 1u << (rel - E) : 0u);
-                const int row = row0 + __popc(starts & ((2u << lane) - 1u));
-                const int64_t c = cv[u];
-                if (c >= cb && c < ce) T[row + (int)(c - cb) * m] = __ldg(values + e0 + E + lane);
+                at[u] = -1;
+                if (E < len) {                                        // warp-uniform
+                    const int row0 = __popc(__ballot_sync(kFull, rel <= E)) - 1;
+                    const unsigned starts =
+                        __reduce_or_sync(kFull, (rel > E && rel < E + 32) ? 1u << (rel - E) : 0u);
+                    const int row = row0 + __popc(starts & ((2u << lane) - 1u));
+                    const int64_t c = cv[u];
+                    if (c >= cb && c < ce) {
+                        at[u] = row + (int)(c - cb) * m;
+                        vv[u] = __ldg(values + e0 + E + lane);
+                    }
+                }
             }
+#pragma unroll
+            for (int u = 0; u < kU; ++u)
+                if (at[u] >= 0) T[at[u]] = vv[u];
         }
         __syncwarp();
         write_tile(out + __ldg(val_off + b), T, np);
