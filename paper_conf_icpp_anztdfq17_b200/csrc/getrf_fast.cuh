@@ -84,14 +84,14 @@ __device__ __forceinline__ unsigned tile_max_key(unsigned key, int t) {
 template <typename R>
 struct FastSmem {
     R slot[64];     // per lane: (a_kk, refined 1/a_kk) -- sub-warp tiles
-    R row[32];      // pivot-row buffer, T elements per tile -- sub-warp tiles
+    R row[2][32];   // pivot-row buffers (alternating steps), T elements per tile
 };
 
 // Compile-time options (defaults chosen by scripts/micro/getrf_bench.cu on the
 // C3 order mix): kFastShflW32 -- full-warp tiles broadcast by SHFL instead of
 // smem; kFastPreRcp -- every lane pre-refines 1/a_kk (shorter chain, more
 // instructions).
-constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4;
+constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4, kFastNoDblBuf = 8;
 #ifndef BJ_FAST_DEFAULT
 #define BJ_FAST_DEFAULT 0
 #endif
@@ -126,6 +126,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     constexpr bool W32 = (T == 32) && ((F & kFastShflW32) != 0);
     constexpr bool PRE = (F & kFastPreRcp) != 0;
     constexpr bool HYB = (T == 32) && !W32 && ((F & kFastHybrid) != 0);
+    constexpr bool DBL = (F & kFastNoDblBuf) == 0;
     const int lane = threadIdx.x & 31;
     const int t = lane / T;
     const int r = lane % T;
@@ -148,13 +149,16 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         tile_ok = false;
     }
     const bool row_ok = tile_ok && (r < M);
-    R *buf = sm.row + tbase;
 
     int tag = row_ok ? 0 : -1;      // 0: candidate; k+1: pivot of step k; -1: inactive lane
     int inf = 0;
     bool redo = false;              // pivot ambiguity or IEEE slow-path quotient in this tile
     static_for<0, M>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
+        // Alternating buffers: step k+1 publishes into the other buffer, so
+        // only the publish -> receive order needs a warp barrier (no barrier
+        // between this step's broadcast loads and the next step's stores).
+        R *buf = sm.row[DBL ? (k & 1) : 0] + tbase;
 #ifdef BJ_TRACE
         if (blockIdx.x == 0 && threadIdx.x == 0) g_ftrace[k] = clock64();
 #endif
@@ -290,7 +294,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                 a[j] = Num<R>::fma(-l, buf[j], a[j]);
             });
         }
-        if constexpr (!W32) __syncwarp();
+        if constexpr (!W32 && !DBL) __syncwarp();
     });
     // Tiles that hit a pivot ambiguity or a slow-path quotient are redone by
     // the safe kernel from the (still untouched) input.

@@ -188,7 +188,7 @@ void run(int64_t nb, const char *name, int force_warps_per_sm = 0) {
     cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
 }
 
-template <typename R>
+template <typename R, bool R2 = true>
 void run_r2(int64_t nb, int LO, int HI, const char *name) {
     std::vector<int64_t> vo(nb + 1), ve(nb + 1);
     std::vector<int32_t> ord(nb);
@@ -226,7 +226,8 @@ void run_r2(int64_t nb, int LO, int HI, const char *name) {
         cudaMemcpy(A, A0, tot * sizeof(R), cudaMemcpyDeviceToDevice);
         cudaMemset(count, 0, 4);
         cudaEventRecord(e0);
-        launch_getrf_r2<R>(A, dvo, dve, piv, info, pv, list, count, 0);
+        if constexpr (R2) launch_getrf_r2<R>(A, dvo, dve, piv, info, pv, list, count, 0);
+        else launch_getrf_fast<R, 17, 32>(A, dvo, dve, piv, info, pv, list, count, 0);
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms; cudaEventElapsedTime(&ms, e0, e1);
@@ -238,8 +239,8 @@ void run_r2(int64_t nb, int LO, int HI, const char *name) {
     for (int64_t i = 0; i < nb; ++i) bytes += 2.0 * sizeof(R) * m_of[i] * m_of[i] + 4 * m_of[i] + 20;
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrf_r2<R>, kR2Threads, r2_dyn_smem(sizeof(R)));
-    printf("R2 sel=%d minb=%d %-22s occ=%d warps/SM  %8.1f us  %7.1f GB/s  %6.1f Mblk/s  deferred=%u err=%s\n",
-           BJ_R2_SELECT, BJ_R2_MINB, name, per_sm * 4, ts[ts.size() / 2] * 1e3, bytes / (ts[ts.size() / 2] * 1e-3) / 1e9,
+    printf("%s sel=%d minb=%d %-22s occ=%d warps/SM  %8.1f us  %7.1f GB/s  %6.1f Mblk/s  deferred=%u err=%s\n",
+           R2 ? "R2" : "F0", BJ_R2_SELECT, BJ_R2_MINB, name, per_sm * 4, ts[ts.size() / 2] * 1e3, bytes / (ts[ts.size() / 2] * 1e-3) / 1e9,
            nb / (ts[ts.size() / 2] * 1e-3) / 1e6, hc, cudaGetErrorString(cudaGetLastError()));
     cudaFree(A); cudaFree(A0); cudaFree(dvo); cudaFree(dve); cudaFree(dbs); cudaFree(dord); cudaFree(piv); cudaFree(info);
     cudaFree(list); cudaFree(count);
@@ -249,18 +250,25 @@ int main(int argc, char **argv) {
 #ifdef BJ_TRACE
     run_fast1<32>(148, "FAST 1 warp");
 #else
+    if (argc > 2) {
+        run_r2<float, false>(552000, 17, 32, "mix 17..32 f32 F0");
+        run_r2<float, true>(552000, 17, 32, "mix 17..32 f32 R2");
+        run_r2<double, false>(552000, 17, 32, "mix 17..32 f64 F0");
+        run_r2<double, true>(552000, 17, 32, "mix 17..32 f64 R2");
+        return 0;
+    }
     if (argc > 1) {
         run_r2<double>(40000, 32, 32, "m=32 f64");
         run_r2<double>(552000, 17, 32, "mix 17..32 f64");
         run_r2<float>(552000, 17, 32, "mix 17..32 f32");
         return 0;
     }
-    run_mix_fast<32, 32, 0>(40000, "m=32 F0 smem");
-    run_mix_fast<32, 32, 4>(40000, "m=32 F4 hybrid");
-    run_mix_fast<32, 32, 6>(40000, "m=32 F6 hybrid+pre");
-    run_mix_fast<17, 32, 0>(552000, "mix FAST F0 smem");
-    run_mix_fast<17, 32, 4>(552000, "mix FAST F4 hybrid");
-    run_mix_fast<17, 32, 6>(552000, "mix FAST F6 hybrid+pre");
+    run_mix_fast<32, 32, 0>(40000, "m=32 F0 dblbuf");
+    run_mix_fast<32, 32, 8>(40000, "m=32 F8 single buf");
+    run_mix_fast<17, 32, 0>(552000, "mix FAST F0 dblbuf");
+    run_mix_fast<17, 32, 8>(552000, "mix FAST F8 single buf");
+    run_mix_fast<9, 16, 0>(276000, "mix9-16 F0 dblbuf");
+    run_mix_fast<9, 16, 8>(276000, "mix9-16 F8 single");
 #endif
     return 0;
 }

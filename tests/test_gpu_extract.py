@@ -66,6 +66,35 @@ def test_random_csr_unsorted(dtype):
         _check(rp, ci, va, np.asarray(edges, np.int32))
 
 
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_empty_rows_and_long_rows(dtype):
+    """Blocks with empty rows (first, last and middle rows of a block: the
+    row-by-row fallback) next to blocks whose rows are longer than several
+    32-entry chunks (the chunked scan, rows crossing chunk and round edges)."""
+    rng = np.random.default_rng(43)
+    n = 2000
+    rows = []
+    for r in range(n):
+        u = rng.random()
+        if u < 0.15:
+            c = np.zeros(0, np.int64)                                 # empty row
+        elif u < 0.3:
+            c = rng.choice(n, size=int(rng.integers(100, 700)), replace=False)   # long row
+        else:
+            c = np.unique(np.clip(r + rng.integers(-40, 41, size=30), 0, n - 1))
+        rng.shuffle(c)
+        rows.append(c)
+    rp = np.concatenate([[0], np.cumsum([len(c) for c in rows])]).astype(np.int64)
+    ci = np.concatenate(rows).astype(np.int32)
+    va = rng.uniform(-1, 1, size=len(ci)).astype(dtype)
+    for b in (1, 5, 16, 32):
+        _check(rp, ci, va, S.uniform_block_ptr(n, b))
+    edges = [0]
+    while edges[-1] < n:
+        edges.append(min(n, edges[-1] + int(rng.integers(1, 33))))
+    _check(rp, ci, va, np.asarray(edges, np.int32))
+
+
 def test_heavy_rows_take_the_cta_path():
     """Rows with far more than kHeavy entries (skewed nnz)."""
     rng = np.random.default_rng(42)

@@ -17,11 +17,14 @@ pytestmark = pytest.mark.gpu
 TOL = {torch.float64: 1e-13, torch.float32: 1e-5}
 
 
-def _run(sizes_np, dtype, kind="uniform", values_np=None, plan=True):
+def _run(sizes_np, dtype, kind="uniform", values_np=None, plan=True, b_np=None):
     npdt = NP[dtype]
     vec, val = host_layout(sizes_np, dtype)
     A = values_np if values_np is not None else S.block_values(sizes_np, val, dtype=npdt, kind=kind)
-    b = S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt) if len(sizes_np) else np.zeros(0, npdt)
+    if b_np is not None:
+        b = b_np
+    else:
+        b = S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt) if len(sizes_np) else np.zeros(0, npdt)
     batch = device_batch(sizes_np, dtype, values_np=A)
     # block boundaries (a1) bit-exact
     assert np.array_equal(batch.vec_off.cpu().numpy(), vec)
@@ -109,6 +112,40 @@ def test_special_matrices():
     for i, B in enumerate(blocks):
         A[val[i]: val[i] + m * m] = B.flatten(order="F")
     _run(sizes, torch.float64, values_np=A)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_extreme_ranges_slow_paths(dtype):
+    """Blocks and right-hand sides scaled to the edges of the exponent range,
+    mixed with ordinary blocks in the same warps (every size class): GETRF
+    defers |a| >= 2^990 / tiny blocks to its exact path, GETRS flags quotients
+    that need the IEEE slow path and redoes only those tiles.  Results stay
+    bit-identical to the oracle (NaN positions included)."""
+    npdt = NP[dtype]
+    big, tiny, sub = (1e300, 1e-300, 1e-310) if dtype == torch.float64 else (1e37, 1e-37, 1e-42)
+    sizes = np.repeat(np.array([3, 7, 13, 24, 32], np.int32), 37)
+    vec, val = host_layout(sizes, dtype)
+    A = S.block_values(sizes, val, dtype=npdt)
+    b = S.rhs_values(sizes, dtype=npdt).copy()
+    for i in range(len(sizes)):
+        m = int(sizes[i])
+        blk = slice(int(val[i]), int(val[i]) + m * m)
+        seg = slice(int(vec[i]), int(vec[i]) + m)
+        kind = i % 6
+        if kind == 1:
+            A[blk] = (A[blk].astype(np.float64) * big).astype(npdt)
+        elif kind == 2:
+            A[blk] = (A[blk].astype(np.float64) * tiny).astype(npdt)
+        elif kind == 3:
+            b[seg] = (b[seg].astype(np.float64) * sub).astype(npdt)     # subnormal right-hand sides
+        elif kind == 4:
+            A[blk] = (A[blk].astype(np.float64) * tiny).astype(npdt)
+            b[seg] = (b[seg].astype(np.float64) * big).astype(npdt)      # quotients overflow
+    r = _run(sizes, dtype, values_np=A, b_np=b)
+    xd, xo = bits(r["x_d"]), bits(r["x_o"])
+    nan_d, nan_o = np.isnan(r["x_d"]), np.isnan(r["x_o"])
+    assert np.array_equal(nan_d, nan_o)
+    assert np.array_equal(xd[~nan_d], xo[~nan_o])
 
 
 def test_padding_invariance_on_device():
