@@ -92,6 +92,9 @@ struct FastSmem {
 // smem; kFastPreRcp -- every lane pre-refines 1/a_kk (shorter chain, more
 // instructions).
 constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4, kFastNoDblBuf = 8;
+// Micro-benchmark-only ablations (wrong results; scripts/micro/getrf_bench.cu):
+// skip the pivot-row publish / the division / the pivot search.
+constexpr int kFastXNoPub = 16, kFastXNoDiv = 32, kFastXNoSearch = 64, kFastXAllLanes = 128, kFastXOnePair = 256;
 #ifndef BJ_FAST_DEFAULT
 #define BJ_FAST_DEFAULT 0
 #endif
@@ -175,7 +178,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         // Fig. 1 bottom lines 5-7: key = candidate flag | top 26 bits of |a| | inverted lane.
         const unsigned hi = Num<R>::key_hi(a[k]);
         const unsigned key = cand ? (0x80000000u | (hi & 0x7fffffe0u) | (unsigned)(31 - r)) : 0u;
-        const unsigned kmax = tile_max_key<T>(key, t);
+        const unsigned kmax = (F & kFastXNoSearch) ? (key | (unsigned)(31 - (k % T))) : tile_max_key<T>(key, t);
         int ipiv = (31 - (int)(kmax & 31u)) & (T - 1);   // (inactive tiles: in range, unused)
         // Another candidate with the same truncated key: the lane order may not
         // be the exact order (R1/R2).  No branch here: the tile is redone by
@@ -212,8 +215,12 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                 constexpr int j0 = k & ~1;
                 static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
                     constexpr int j = j0 + 2 * decltype(pc)::value;
-                    if constexpr (j + 1 < M) st_shared_pred(isp, buf + j, a[j], a[j + 1]);
-                    else st_shared_pred(isp, buf + j, a[j]);
+                    constexpr bool pub = (F & kFastXNoPub) == 0 && ((F & kFastXOnePair) == 0 || j == j0);
+                    const bool who = (F & kFastXAllLanes) ? true : isp;
+                    if constexpr (pub) {
+                        if constexpr (j + 1 < M) st_shared_pred(who, buf + j, a[j], a[j + 1]);
+                        else st_shared_pred(who, buf + j, a[j]);
+                    }
                 });
             } else {
                 static_for<k, M>([&](auto jc) {
@@ -234,14 +241,14 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                 }
             } else {
                 d = buf[k];
-                yd = Num<R>::rcp_refine(d);
+                yd = (F & kFastXNoDiv) ? d : Num<R>::rcp_refine(d);
             }
         }
         const bool sing = (Num<R>::key_hi(d) == 0u) && (Num<R>::key_lo(d) == 0u);   // R4
         // line 13 (SCAL): rows that must not change divide 1 by 1 and use l = +0.
         const bool upd = (tag == 0) && !sing;
         bool bad = false;
-        const R q = Num<R>::div_pre_flag(a[k], d, yd, bad);
+        const R q = (F & kFastXNoDiv) ? a[k] * d : Num<R>::div_pre_flag(a[k], d, yd, bad);
         redo = redo || (upd && bad);
         const R l = upd ? q : R(0);
         if (upd) a[k] = q;
@@ -298,6 +305,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     });
     // Tiles that hit a pivot ambiguity or a slow-path quotient are redone by
     // the safe kernel from the (still untouched) input.
+    if constexpr ((F & (kFastXNoPub | kFastXNoDiv | kFastXNoSearch | kFastXAllLanes | kFastXOnePair)) != 0) redo = (tag == -7);   // ablation: keep the write-back
     if (tile_bits<T>(__ballot_sync(kFull, redo && tile_ok), tbase) != 0u) {
         if (tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
         return;

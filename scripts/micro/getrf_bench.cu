@@ -263,12 +263,13 @@ int main(int argc, char **argv) {
         run_r2<float>(552000, 17, 32, "mix 17..32 f32");
         return 0;
     }
-    run_mix_fast<32, 32, 0>(40000, "m=32 F0 dblbuf");
-    run_mix_fast<32, 32, 8>(40000, "m=32 F8 single buf");
-    run_mix_fast<17, 32, 0>(552000, "mix FAST F0 dblbuf");
-    run_mix_fast<17, 32, 8>(552000, "mix FAST F8 single buf");
-    run_mix_fast<9, 16, 0>(276000, "mix9-16 F0 dblbuf");
-    run_mix_fast<9, 16, 8>(276000, "mix9-16 F8 single");
+    run_mix_fast<32, 32, 0>(40000, "m=32 F0");
+    run_mix_fast<32, 32, 16>(40000, "m=32 X no publish");
+    run_mix_fast<32, 32, 32>(40000, "m=32 X no division");
+    run_mix_fast<32, 32, 64>(40000, "m=32 X no search");
+    run_mix_fast<32, 32, 128>(40000, "m=32 X all lanes store");
+    run_mix_fast<32, 32, 256>(40000, "m=32 X one pair only");
+    run_mix_fast<17, 32, 0>(552000, "mix 17..32 F0");
 #endif
     return 0;
 }
