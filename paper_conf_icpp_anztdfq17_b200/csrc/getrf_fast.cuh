@@ -91,7 +91,7 @@ struct FastSmem {
 // C3 order mix): kFastShflW32 -- full-warp tiles broadcast by SHFL instead of
 // smem; kFastPreRcp -- every lane pre-refines 1/a_kk (shorter chain, more
 // instructions).
-constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4, kFastNoDblBuf = 8;
+constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4, kFastDblBuf = 8;
 // Micro-benchmark-only ablations (wrong results; scripts/micro/getrf_bench.cu):
 // skip the pivot-row publish / the division / the pivot search.
 constexpr int kFastXNoPub = 16, kFastXNoDiv = 32, kFastXNoSearch = 64, kFastXAllLanes = 128, kFastXOnePair = 256;
@@ -129,7 +129,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     constexpr bool W32 = (T == 32) && ((F & kFastShflW32) != 0);
     constexpr bool PRE = (F & kFastPreRcp) != 0;
     constexpr bool HYB = (T == 32) && !W32 && ((F & kFastHybrid) != 0);
-    constexpr bool DBL = (F & kFastNoDblBuf) == 0;
+    constexpr bool DBL = (F & kFastDblBuf) != 0;
     const int lane = threadIdx.x & 31;
     const int t = lane / T;
     const int r = lane % T;
