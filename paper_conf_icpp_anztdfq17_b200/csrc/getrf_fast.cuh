@@ -222,6 +222,19 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                         else st_shared_pred(who, buf + j, a[j]);
                     }
                 });
+            } else if constexpr (sizeof(R) == 4 && T >= 4) {
+                // fp32: 16-B quads (4x fewer one-lane stores than scalars)
+                constexpr int j0 = k & ~3;
+                static_for<0, (M - j0 + 3) / 4>([&](auto pc) {
+                    constexpr int j = j0 + 4 * decltype(pc)::value;
+                    if constexpr (j + 3 < M) {
+                        st_shared_pred(isp, buf + j, a[j], a[j + 1], a[j + 2], a[j + 3]);
+                    } else {
+                        if constexpr (j + 1 < M) st_shared_pred(isp, buf + j, a[j], a[j + 1]);
+                        else st_shared_pred(isp, buf + j, a[j]);
+                        if constexpr (j + 2 < M) st_shared_pred(isp, buf + j + 2, a[j + 2]);
+                    }
+                });
             } else {
                 static_for<k, M>([&](auto jc) {
                     constexpr int j = decltype(jc)::value;
@@ -293,6 +306,27 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                     a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
                 } else {
                     a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                }
+            });
+        } else if constexpr (sizeof(R) == 4 && T >= 4) {
+            constexpr int g0 = (k + 4) & ~3;            // first quad after column k
+            static_for<k + 1, (g0 < M ? g0 : M)>([&](auto jc) {
+                constexpr int j = decltype(jc)::value;
+                a[j] = Num<R>::fma(-l, buf[j], a[j]);
+            });
+            static_for<0, (g0 < M ? (M - g0 + 3) / 4 : 0)>([&](auto pc) {
+                constexpr int j = g0 + 4 * decltype(pc)::value;
+                if constexpr (j + 3 < M) {
+                    const float4 u = *reinterpret_cast<const float4 *>(buf + j);
+                    a[j] = Num<R>::fma(-l, u.x, a[j]);
+                    a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
+                    a[j + 2] = Num<R>::fma(-l, u.z, a[j + 2]);
+                    a[j + 3] = Num<R>::fma(-l, u.w, a[j + 3]);
+                } else {
+                    static_for<j, M>([&](auto jc) {
+                        constexpr int jj = decltype(jc)::value;
+                        a[jj] = Num<R>::fma(-l, buf[jj], a[jj]);
+                    });
                 }
             });
         } else {
