@@ -31,7 +31,7 @@ import torch.distributed as dist
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22)}   # per-GPU z-slab of 22 planes
+FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22), "SV": (174, 174, 22)}   # per-GPU z-slab of 22 planes
 
 CONFIGS = {
     # name: (nblocks per GPU, lo, hi, dtype, description)
@@ -41,6 +41,7 @@ CONFIGS = {
     "C1": (1_000, 4, 16, torch.float64, "C1: 1,000 blocks m ~ U{4..16}, fp64 (latency case, L2-resident)"),
     "C4": (0, 24, 24, torch.float64, "C4: diagonal-block extraction, 27-pt x 3-dof FEM CSR, 1,998,216 rows/GPU, skewed hubs"),
     "C5": (0, 24, 24, torch.float64, "C5: block-Jacobi setup (extract + getrf) + 100 applies, 1,998,216 rows/GPU, b = 24"),
+    "SV": (0, 24, 24, torch.float64, "SV (NEXT 2): supervariable blocking of the C4 CSR pattern, 1,998,216 rows/GPU, bound 24"),
 }
 
 
@@ -416,8 +417,13 @@ def run_fem(args, ws, rank, local):
     h = bj.Handle() if args.config == "C5" else None
     napply = 100
 
+    sv_bytes = 8 * (n + 1) + 4 * A.col_idx.numel() + 4 * (n // b + 2)   # row_ptr + col_idx read, block_ptr written
+    sv_nb = [0]
+
     def step(evs=None):
-        if args.config == "C4":
+        if args.config == "SV":
+            sv_nb[0] = bj.supervariable_blocking(A, b).numel() - 1
+        elif args.config == "C4":
             bj.extract(A, bp, out)
         else:
             if evs is not None:
@@ -449,7 +455,17 @@ def run_fem(args, ws, rank, local):
     line = {"n_gpus": ws, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (counter-based FEM CSR generated on device)",
             "gpu_launches": launches, "clocks": sampler.summary()}
-    if args.config == "C4":
+    if args.config == "SV":
+        achieved = sv_bytes / (ms * 1e-3) / 1e9
+        line.update({"metric": "matrix rows blocked per second", "value": n * ws / (ms * 1e-3),
+                     "unit": "rows/s", "higher_is_better": True,
+                     "config": {"workload": CONFIGS["SV"][4], "bound": b, "rows_per_gpu": n,
+                                "nnz_per_gpu": A.col_idx.numel(), "blocks": sv_nb[0],
+                                "l2": "col_idx (0.62 GB) larger than L2"},
+                     "roofline": {"bound": "hbm", "kernel": "bj_supervariable_blocking (all launches)",
+                                  "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+                                  "traffic": None, "peak_source": peak_src, "bytes_per_launch": sv_bytes}})
+    elif args.config == "C4":
         achieved = ext_bytes / (ms * 1e-3) / 1e9
         line.update({"metric": "diagonal blocks extracted per second", "value": nb * ws / (ms * 1e-3),
                      "unit": "blocks/s", "higher_is_better": True,

@@ -189,6 +189,26 @@ bj_status bj_destroy(bj_handle *handle);
 bj_status bj_partition(int64_t nblocks, const int32_t *sizes_h, int G, int64_t *bounds_h);
 
 /* ---------------------------------------------------------------------------
+ * Next row NEXT(2) -- supervariable blocking (section II.A, P:186-193;
+ * the experiments vary only the upper bound): the block
+ * boundaries that bj_extract takes as input.
+ *   A supervariable is a maximal run of consecutive rows whose column index
+ *   sequences are identical as stored (R20); a supervariable longer than
+ *   `max_block` is cut into max_block-row pieces plus a remainder (R22); the
+ *   pieces are clustered greedily in row order into blocks of at most
+ *   `max_block` rows (R21).  Only A->row_ptr / A->col_idx are read (values
+ *   and dtype are ignored).
+ *   block_ptr: DEVICE int32[A->nrows + 1] (capacity); receives nb+1 entries,
+ *   block_ptr[0] = 0, block_ptr[nb] = nrows.  nblocks_h: HOST int64, receives
+ *   nb.  max_block must lie in 1..32 and nrows in 0..2^31-2, else BJ_ERR_ARG.
+ *   SYNCHRONOUS: returns after the stream work completes (the greedy chain is
+ *   iterated to a fixpoint with a host-read convergence flag; this is a
+ *   once-per-sparsity-pattern analysis, not on the setup/apply path).
+ * ------------------------------------------------------------------------- */
+bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t *block_ptr,
+                                    int64_t *nblocks_h, bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
  * End-to-end call with HOST buffers (synchronous): copies sizes_h (nblocks),
  * blocks_h (nvalues elements, packed per bj_layout) and b_h (nvec elements)
  * to the device, runs layout + plan + GETRF + GETRS, and copies x_h (nvec),

@@ -26,7 +26,7 @@ EXPORTS = (
     "bj_status_string", "bj_version", "bj_layout", "bj_layout_from_block_ptr", "bj_plan_create",
     "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_create", "bj_setup",
     "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
-    "bj_launch_count", "bj_launch_count_reset",
+    "bj_launch_count", "bj_launch_count_reset", "bj_supervariable_blocking",
     "bj_synth_sizes", "bj_synth_blocks", "bj_synth_rhs", "bj_synth_fem_row_ptr", "bj_synth_fem_fill",
 )
 
@@ -73,6 +73,7 @@ def lib() -> ctypes.CDLL:
             "bj_apply": ([P, P, P, P], I32),
             "bj_destroy": ([P], I32),
             "bj_partition": ([I64, P, I32, P], I32),
+            "bj_supervariable_blocking": ([P, I32, P, P, P], I32),
             "bj_workspace_create": ([P], I32),
             "bj_workspace_destroy": ([P], I32),
             "bj_gesv_host": ([P, I64, P, I64, P, I64, P, P, P, P, I32, P], I32),
@@ -265,6 +266,18 @@ class Handle:
             self.close()
         except Exception:
             pass
+
+
+def supervariable_blocking(A: Csr, max_block: int, stream=None) -> torch.Tensor:
+    """NEXT(2): block_ptr (int32 device tensor [nb+1]) of supervariable
+    blocking with upper bound `max_block` (R20-R22).  Synchronous."""
+    n = A.row_ptr.numel() - 1
+    bp = torch.empty(n + 1, dtype=torch.int32, device=A.row_ptr.device)
+    nb = ctypes.c_int64(0)
+    a = A.c()
+    _check(lib().bj_supervariable_blocking(ctypes.byref(a), int(max_block), _p(bp), ctypes.byref(nb),
+                                           _stream(stream)), "bj_supervariable_blocking")
+    return bp[: nb.value + 1]
 
 
 def partition(sizes: np.ndarray, G: int) -> np.ndarray:

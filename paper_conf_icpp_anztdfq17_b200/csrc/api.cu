@@ -164,6 +164,15 @@ bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out, b
     return extract_run<float>(*A, block_ptr, out->nblocks, out->val_off, (float *)out->values, s);
 }
 
+bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t *block_ptr, int64_t *nblocks_h,
+                                    bj_stream_t stream) {
+    pool_keep_memory();
+    if (!A || !block_ptr || !nblocks_h || max_block < 1 || max_block > kMaxM) return BJ_ERR_ARG;
+    if (A->nrows < 0 || A->nrows > 2147483646LL || A->nnz < 0 || !A->row_ptr) return BJ_ERR_ARG;
+    if (A->nnz > 0 && !A->col_idx) return BJ_ERR_ARG;
+    return supervariable_run(*A, max_block, block_ptr, nblocks_h, (cudaStream_t)stream);
+}
+
 bj_status bj_getrf_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const bj_plan *plan,
                             bj_stream_t stream) {
     pool_keep_memory();

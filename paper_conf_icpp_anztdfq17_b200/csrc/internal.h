@@ -32,4 +32,8 @@ template <typename R>
 bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, const int64_t *val_off,
                       R *out, cudaStream_t s);
 
+// NEXT(2)
+bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, int64_t *nblocks_h,
+                            cudaStream_t s);
+
 }  // namespace bj
