@@ -73,7 +73,7 @@ __global__ void k_unit_pos(const int32_t *__restrict__ svstart, int32_t n, int32
 // entry[t]; the first node >= the segment end is the entry of segment t+1.
 // write == nullptr: fixpoint pass (counts + exits); else write the nodes.
 __global__ void k_sv_walk(const int32_t *__restrict__ prevB, int32_t n, int32_t bound, int32_t nseg,
-                          const int32_t *__restrict__ entry, int32_t *__restrict__ entry_next,
+                          const int32_t *entry, int32_t *entry_next,   // may alias (in-place pass)
                           int32_t *__restrict__ count, int32_t *__restrict__ changed,
                           const int32_t *__restrict__ off, int32_t *__restrict__ block_ptr) {
     const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
