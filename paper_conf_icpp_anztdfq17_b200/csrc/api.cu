@@ -166,10 +166,10 @@ bj_status bj_extract(const bj_csr *A, const int32_t *block_ptr, bj_batch *out, b
 
 bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t *block_ptr, int64_t *nblocks_h,
                                     bj_stream_t stream) {
-    pool_keep_memory();
     if (!A || !block_ptr || !nblocks_h || max_block < 1 || max_block > kMaxM) return BJ_ERR_ARG;
     if (A->nrows < 0 || A->nrows > 2147483646LL || A->nnz < 0 || !A->row_ptr) return BJ_ERR_ARG;
     if (A->nnz > 0 && !A->col_idx) return BJ_ERR_ARG;
+    pool_keep_memory();
     return supervariable_run(*A, max_block, block_ptr, nblocks_h, (cudaStream_t)stream);
 }
 

@@ -80,3 +80,10 @@ def test_errors_without_gpu_are_arguments(lib):
     assert lib.bj_layout(4, None, 7, None, None, None) == -1
     lib.bj_partition.argtypes = [ctypes.c_int64, ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p]
     assert lib.bj_partition(3, None, 0, None) == -1
+    lib.bj_supervariable_blocking.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                              ctypes.c_void_p]
+    assert lib.bj_supervariable_blocking(None, 8, None, None, None) == -1
+    csr = (ctypes.c_int64 * 8)(4, 0, 0, 0, 0, 0, 0, 0)          # nrows = 4, row_ptr = NULL
+    nb = ctypes.c_int64(0)
+    assert lib.bj_supervariable_blocking(ctypes.cast(csr, ctypes.c_void_p), 33, ctypes.c_void_p(16), ctypes.byref(nb),
+                                         None) == -1
