@@ -17,14 +17,20 @@
 //   3. k_unit_pos: unit boundary at i iff (i - svstart[i]) % bound == 0 (R22);
 //      unit[n] = n.  Inclusive max-scan -> prevB[x] = largest boundary <= x.
 //   4. The greedy walk (R21) is the chain p -> next(p) = prevB[min(p+bound, n)]
-//      from p = 0 (every unit has <= bound rows, so next(p) > p).  The rows
-//      are cut into segments of kSegRows; one thread walks each segment from
-//      a guessed entry node, and the exit node of segment t becomes the entry
-//      of t+1.  Iterated to a fixpoint (entry[0] = 0 is exact, so by induction
-//      the fixpoint is the true chain; chains from different starts merge
-//      quickly because next() is monotone, so 2 passes are typical).
-//   5. exclusive sum of per-segment node counts, then each segment writes its
-//      nodes into block_ptr.
+//      from p = 0 (every unit has <= bound rows, so next(p) > p).  Rows are cut
+//      into segments of kSegRows.  The chain enters segment t at an offset
+//      e in [0, bound) (the previous node is < t*kSegRows and next() advances
+//      at most `bound` rows), so k_sv_table lets lane e of warp t walk the
+//      segment from t*kSegRows + e and record (exit offset, node count): the
+//      segment's transfer function for every possible entry.
+//   5. k_sv_compose (one CTA) composes the transfer functions in row order
+//      from entry 0 -- a table lookup per segment, staged through shared
+//      memory -- giving each segment's true entry and node count.  (Chains
+//      from different starts need not merge -- uniform 3-row supervariables
+//      give parallel chains -- so guessing entries and iterating is O(nseg)
+//      passes; the tables make it one pass.)
+//   6. exclusive sum of the per-segment counts, then each segment re-walks
+//      from its entry and writes its nodes into block_ptr.
 #include <cub/cub.cuh>
 
 #include "common.cuh"
@@ -34,7 +40,8 @@ namespace bj {
 
 namespace {
 
-constexpr int kSegRows = 512;
+constexpr int kSegRows = 2048;
+constexpr int kComposeSegs = 256;   // segments staged per shared-memory chunk
 constexpr int kFlagThreads = 256;
 
 struct MaxI32 {
@@ -69,43 +76,62 @@ __global__ void k_unit_pos(const int32_t *__restrict__ svstart, int32_t n, int32
         unit[i] = (i == n || ((int32_t)i - svstart[i]) % bound == 0) ? (int32_t)i : 0;
 }
 
-// Segment t covers rows [t*kSegRows, (t+1)*kSegRows).  Walks the chain from
-// entry[t]; the first node >= the segment end is the entry of segment t+1.
-// write == nullptr: fixpoint pass (counts + exits); else write the nodes.
+// Segment t covers rows [t*kSegRows, (t+1)*kSegRows): write the chain nodes
+// from its entry at off[t]; the last segment appends block_ptr[nb] = n.
 __global__ void k_sv_walk(const int32_t *__restrict__ prevB, int32_t n, int32_t bound, int32_t nseg,
-                          const int32_t *entry, int32_t *entry_next,   // may alias (in-place pass)
-                          int32_t *__restrict__ count, int32_t *__restrict__ changed,
-                          const int32_t *__restrict__ off, int32_t *__restrict__ block_ptr) {
+                          const int32_t *__restrict__ entry, const int32_t *__restrict__ off,
+                          int32_t *__restrict__ block_ptr) {
     const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= nseg) return;
     const int64_t end64 = (int64_t)(t + 1) * kSegRows;
     const int32_t end = end64 < n ? (int32_t)end64 : n;
     int32_t p = entry[t], c = 0;
-    int32_t *dst = block_ptr ? block_ptr + off[t] : nullptr;
+    int32_t *dst = block_ptr + off[t];
     while (p < end) {
-        if (dst) dst[c] = p;
+        dst[c++] = p;
+        const int64_t q = (int64_t)p + bound;
+        p = prevB[q < n ? q : n];
+    }
+    if (t == nseg - 1) dst[c] = n;
+}
+
+// Lane e of warp t walks segment t from row t*kSegRows + e (e < bound);
+// table[t*32 + e] = (node count << 8) | exit offset into segment t+1.
+__global__ void k_sv_table(const int32_t *__restrict__ prevB, int32_t n, int32_t bound, int32_t nseg,
+                           int32_t *__restrict__ table) {
+    const int lane = threadIdx.x & 31;
+    const int64_t t = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (t >= nseg || lane >= bound) return;
+    const int64_t base = t * kSegRows, end64 = base + kSegRows;
+    const int32_t end = end64 < n ? (int32_t)end64 : n;
+    int32_t p = (int32_t)(base + lane), c = 0;
+    while (p < end) {
         ++c;
         const int64_t q = (int64_t)p + bound;
         p = prevB[q < n ? q : n];
     }
-    if (!block_ptr) {
-        count[t] = c;
-        if (t + 1 < nseg) {
-            if (entry_next[t + 1] != p) { entry_next[t + 1] = p; *changed = 1; }
-        }
-    } else if (t == nseg - 1) {
-        block_ptr[off[t] + c] = n;
-    }
+    table[t * 32 + lane] = (c << 8) | (int32_t)(p - end);   // p - end < bound
 }
 
-// Initial guess of segment entries: a boundary node in [t*kSegRows, +bound].
-__global__ void k_sv_guess(const int32_t *__restrict__ prevB, int32_t n, int32_t bound, int32_t nseg,
-                           int32_t *__restrict__ entry) {
-    const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= nseg) return;
-    if (t == 0) { entry[0] = 0; return; }
-    const int64_t q = (int64_t)t * kSegRows + bound;
-    entry[t] = prevB[q < n ? q : n];
+// One CTA: compose the segment transfer functions from entry offset 0.
+__global__ void k_sv_compose(const int32_t *__restrict__ table, int32_t nseg, int32_t *__restrict__ entry,
+                             int32_t *__restrict__ count) {
+    __shared__ int32_t tab[kComposeSegs * 32];
+    int32_t e = 0;   // valid in thread 0
+    for (int64_t t0 = 0; t0 < nseg; t0 += kComposeSegs) {
+        const int32_t nt = (int32_t)((nseg - t0) < kComposeSegs ? (nseg - t0) : kComposeSegs);
+        __syncthreads();
+        for (int i = threadIdx.x; i < nt * 32; i += blockDim.x) tab[i] = table[t0 * 32 + i];
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int32_t k = 0; k < nt; ++k) {
+                const int32_t v = tab[k * 32 + e];
+                entry[t0 + k] = (int32_t)((t0 + k) * kSegRows) + e;
+                count[t0 + k] = v >> 8;
+                e = v & 0xff;
+            }
+        }
+    }
 }
 
 }  // namespace
@@ -120,7 +146,7 @@ bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, 
         return BJ_OK;
     }
     const int32_t nseg = (int32_t)((n + (int64_t)kSegRows - 1) / kSegRows);
-    // scratch: svpos/unit [n+1], svstart/prevB [n+1], entry, count, off [nseg], changed
+    // scratch: svpos/unit/table [n+1], svstart/prevB [n+1], entry, count, off [nseg]
     size_t scan_bytes = 0, sum_bytes = 0;
     cub::DeviceScan::InclusiveScan(nullptr, scan_bytes, (int32_t *)nullptr, (int32_t *)nullptr, MaxI32(), n + 1, s);
     cub::DeviceScan::ExclusiveSum(nullptr, sum_bytes, (int32_t *)nullptr, (int32_t *)nullptr, nseg, s);
@@ -134,10 +160,9 @@ bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, 
     int32_t *entry = reinterpret_cast<int32_t *>(scratch + 2 * vec_bytes);
     int32_t *count = reinterpret_cast<int32_t *>(scratch + 2 * vec_bytes + seg_bytes);
     int32_t *off = reinterpret_cast<int32_t *>(scratch + 2 * vec_bytes + 2 * seg_bytes);
-    int32_t *changed = reinterpret_cast<int32_t *>(scratch + 2 * vec_bytes + 3 * seg_bytes);
     void *tmp = scratch + 2 * vec_bytes + 3 * seg_bytes + 256;
     bj_status st = BJ_OK;
-    int32_t h_changed = 1, h_last[2] = {0, 0};
+    int32_t h_last[2] = {0, 0};
     const int grid = 4 * sm_count();
     const int sgrid = (nseg + 127) / 128;
 
@@ -147,22 +172,14 @@ bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, 
     k_unit_pos<<<grid, 256, 0, s>>>(b, n, bound, a);
     BJ_LAUNCH_CHECK();
     if (cub::DeviceScan::InclusiveScan(tmp, scan_bytes, a, b, MaxI32(), n + 1, s) != cudaSuccess) st = BJ_ERR_CUDA;
-    k_sv_guess<<<sgrid, 128, 0, s>>>(b, n, bound, nseg, entry);
+    k_sv_table<<<(int)(((int64_t)nseg * 32 + 127) / 128), 128, 0, s>>>(b, n, bound, nseg, a);
     BJ_LAUNCH_CHECK();
-    for (int it = 0; st == BJ_OK && h_changed && it <= nseg; ++it) {
-        if (cudaMemsetAsync(changed, 0, sizeof(int32_t), s) != cudaSuccess) { st = BJ_ERR_CUDA; break; }
-        // entries are updated in place: a pass may read an entry a neighbour
-        // just fixed, which only speeds convergence; the fixpoint is the same.
-        k_sv_walk<<<sgrid, 128, 0, s>>>(b, n, bound, nseg, entry, entry, count, changed, nullptr, nullptr);
-        BJ_LAUNCH_CHECK();
-        if (cudaMemcpyAsync(&h_changed, changed, sizeof(int32_t), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
-            cudaStreamSynchronize(s) != cudaSuccess) { st = BJ_ERR_CUDA; break; }
-    }
+    k_sv_compose<<<1, 1024, 0, s>>>(a, nseg, entry, count);
+    BJ_LAUNCH_CHECK();
+    if (st == BJ_OK && cub::DeviceScan::ExclusiveSum(tmp, sum_bytes, count, off, nseg, s) != cudaSuccess)
+        st = BJ_ERR_CUDA;
     if (st == BJ_OK) {
-        if (cub::DeviceScan::ExclusiveSum(tmp, sum_bytes, count, off, nseg, s) != cudaSuccess) st = BJ_ERR_CUDA;
-    }
-    if (st == BJ_OK) {
-        k_sv_walk<<<sgrid, 128, 0, s>>>(b, n, bound, nseg, entry, entry, count, changed, off, block_ptr);
+        k_sv_walk<<<sgrid, 128, 0, s>>>(b, n, bound, nseg, entry, off, block_ptr);
         BJ_LAUNCH_CHECK();
         if (cudaMemcpyAsync(&h_last[0], off + (nseg - 1), sizeof(int32_t), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
             cudaMemcpyAsync(&h_last[1], count + (nseg - 1), sizeof(int32_t), cudaMemcpyDeviceToHost, s) !=
