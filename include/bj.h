@@ -201,9 +201,9 @@ bj_status bj_partition(int64_t nblocks, const int32_t *sizes_h, int G, int64_t *
  *   block_ptr: DEVICE int32[A->nrows + 1] (capacity); receives nb+1 entries,
  *   block_ptr[0] = 0, block_ptr[nb] = nrows.  nblocks_h: HOST int64, receives
  *   nb.  max_block must lie in 1..32 and nrows in 0..2^31-2, else BJ_ERR_ARG.
- *   SYNCHRONOUS: returns after the stream work completes (the greedy chain is
- *   iterated to a fixpoint with a host-read convergence flag; this is a
- *   once-per-sparsity-pattern analysis, not on the setup/apply path).
+ *   SYNCHRONOUS: returns after the stream work completes (nb is read back to
+ *   the host; this is a once-per-sparsity-pattern analysis, not on the
+ *   setup/apply path).
  * ------------------------------------------------------------------------- */
 bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t *block_ptr,
                                     int64_t *nblocks_h, bj_stream_t stream);
