@@ -60,10 +60,11 @@ __global__ void k_sv_flags(const int64_t *__restrict__ row_ptr, const int32_t *_
             if (len != a1 - a0) {
                 start = true;
             } else {
-                for (int64_t k = lane; k - lane < len; k += 32) {
-                    const bool diff = k < len && col_idx[a0 + k] != col_idx[a1 + k];
-                    if (__any_sync(kFull, diff)) { start = true; break; }
-                }
+                // no early exit: every chunk's loads are independent and in flight together
+                bool diff = false;
+#pragma unroll 4
+                for (int64_t k = lane; k < len; k += 32) diff |= __ldg(col_idx + a0 + k) != __ldg(col_idx + a1 + k);
+                start = __any_sync(kFull, diff);
             }
         }
         if (lane == 0) svpos[i] = start ? (int32_t)i : 0;
@@ -163,7 +164,7 @@ bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, 
     void *tmp = scratch + 2 * vec_bytes + 3 * seg_bytes + 256;
     bj_status st = BJ_OK;
     int32_t h_last[2] = {0, 0};
-    const int grid = 4 * sm_count();
+    const int grid = 8 * sm_count();   // 64 warps per SM for the latency-bound row compare
     const int sgrid = (nseg + 127) / 128;
 
     k_sv_flags<<<grid, kFlagThreads, 0, s>>>(A.row_ptr, A.col_idx, n, a);
