@@ -3,15 +3,17 @@
 triangular solves on B200, one process per GPU.
 
 Default workload (BASELINE.json metric, north-star target): config C3 -- 1M
-blocks per GPU with orders m ~ U{4..32}, fp64.  A *step* is one pass of the
-whole hot path over one batch: layout (a1) + size plan + GETRF (a3) + GETRS
-(a4).  Each step factors its own pristine copy of the batch (generated before
-the timed region; 3.2 GB >> 126 MB L2, so no L2 flush is needed).
+blocks with orders m ~ U{4..32}, fp64.  A *step* is one pass of the whole hot
+path over one batch: layout (a1) + size plan + GETRF (a3) + GETRS (a4).  Each
+step factors its own pristine copy of the batch (generated before the timed
+region; 3.2 GB >> 126 MB L2, so no L2 flush is needed).
 
-Multi-GPU (torchrun, NCCL): the global batch of N x 1M blocks is split by the
-contiguous cost-balanced partitioner (row a6); ranks regenerate their shard
-from the counter generator; no collective on the data path; barrier + max
-over ranks of the CUDA-event time.
+Multi-GPU (one process per GPU, NCCL): ``--gpus N`` started as a plain process
+re-launches itself under torch.distributed.run.  The batch (C3: 1M blocks) is
+split by the contiguous cost-balanced partitioner (row a6) -- strong scaling
+(``--scaling weak`` replicates the per-GPU batch instead); ranks regenerate
+their shard from the counter generator; no collective on the data path;
+barrier + max over ranks of the CUDA-event time.
 
 ``--impl reference`` times the CPU oracle (the reference arm of this tier).
 """
@@ -35,9 +37,9 @@ FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22), "SV": (174, 174, 22)}   # per
 
 CONFIGS = {
     # name: (nblocks per GPU, lo, hi, dtype, description)
-    "C3": (1_000_000, 4, 32, torch.float64, "C3: 1M blocks/GPU, m ~ U{4..32}, fp64, LU + solve"),
-    "C3f32": (1_000_000, 4, 32, torch.float32, "C3: 1M blocks/GPU, m ~ U{4..32}, fp32, LU + solve"),
-    "C2": (40_000, 32, 32, torch.float64, "C2: 40,000 blocks 32x32/GPU, fp64, LU + solve"),
+    "C3": (1_000_000, 4, 32, torch.float64, "C3: 1M blocks (sharded over the GPUs), m ~ U{4..32}, fp64, LU + solve"),
+    "C3f32": (1_000_000, 4, 32, torch.float32, "C3: 1M blocks (sharded over the GPUs), m ~ U{4..32}, fp32, LU + solve"),
+    "C2": (40_000, 32, 32, torch.float64, "C2: 40,000 blocks 32x32, fp64, LU + solve"),
     "C1": (1_000, 4, 16, torch.float64, "C1: 1,000 blocks m ~ U{4..16}, fp64 (latency case, L2-resident)"),
     "C4": (0, 24, 24, torch.float64, "C4: diagonal-block extraction, 27-pt x 3-dof FEM CSR, 1,998,216 rows/GPU, skewed hubs"),
     "C5": (0, 24, 24, torch.float64, "C5: block-Jacobi setup (extract + getrf) + 100 applies, 1,998,216 rows/GPU, b = 24"),
@@ -154,53 +156,120 @@ def max_over_ranks(v: float, ws: int) -> float:
     return float(t.item())
 
 
+METRIC = "blocks/s (batched LU + solve)"
+
+
+def workload(args, ws):
+    """(nblocks_total, lo, hi, dtype, description, scaling) of the batched
+    configs.  Multi-GPU default: STRONG scaling -- the config's batch (C3: 1M
+    blocks) is sharded over the ranks by the partitioner (row a6); with
+    --scaling weak every rank gets the full per-GPU batch instead."""
+    nb, lo, hi, dt, desc = CONFIGS[args.config]
+    if args.nblocks:
+        nb = args.nblocks
+    scaling = "weak" if (args.scaling == "weak" and ws > 1) else "strong"
+    nb_total = nb * ws if scaling == "weak" else nb
+    return nb_total, lo, hi, dt, desc, scaling
+
+
 # --------------------------------------------------------------------------
 # CPU oracle timing (cpu_baseline leg and --impl reference)
 # --------------------------------------------------------------------------
-def oracle_sample(nb_target: int, lo: int, hi: int, dt, budget_s: float, first: int = 0):
-    """Time oracle GETRF+GETRS on the first blocks of the workload (same
-    generator), growing the sample in chunks until ~budget_s of CPU work."""
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_data(nb: int, lo: int, hi: int, dt, first: int = 0):
+    """The first nb blocks of the workload (same counter generator as the GPU
+    arm), generated with the C generator (bj_synth/fastgen.c)."""
     import bj_synth as S
     import oracle
     npdt = np.float64 if dt == torch.float64 else np.float32
-    chunk = 20000 if hi > 16 else 100000
-    done, t_total = 0, 0.0
-    while done < nb_target and t_total < budget_s:
-        n = min(chunk, nb_target - done)
-        sizes = S.block_sizes(n, lo, hi, first=first + done)
-        vec, val = oracle.layout(sizes, esize(dt))
-        A = S.block_values(sizes, val, first=first + done, dtype=npdt)
-        b = S.rhs_values(sizes, first=first + done, dtype=npdt)
-        t0 = time.perf_counter()
-        LU, piv, info = oracle.getrf_batch(sizes, val, vec, A)
-        oracle.getrs_batch(sizes, val, vec, LU, piv, b)
-        t_total += time.perf_counter() - t0
-        done += n
-    return done, t_total, oracle.max_threads()
+    sizes = S.block_sizes(nb, lo, hi, first=first)
+    vec, val = oracle.layout(sizes, esize(dt))
+    A = S.block_values_fast(sizes, val, first=first, dtype=npdt)
+    b = S.rhs_values_fast(sizes, first=first, dtype=npdt)
+    return sizes, vec, val, A, b
+
+
+def oracle_run(data, nthreads: int = 0):
+    """One oracle GETRF + GETRS pass over `data`; returns (t_getrf, t_getrs) in s."""
+    import oracle
+    sizes, vec, val, A, b = data
+    t0 = time.perf_counter()
+    LU, piv, info = oracle.getrf_batch(sizes, val, vec, A, nthreads=nthreads)
+    t1 = time.perf_counter()
+    oracle.getrs_batch(sizes, val, vec, LU, piv, b, nthreads=nthreads)
+    t2 = time.perf_counter()
+    return t1 - t0, t2 - t1
+
+
+def oracle_sample_size(nb_max: int, lo: int, hi: int, dt, seconds: float, nthreads: int = 0) -> int:
+    """Blocks of the workload the oracle handles in about `seconds`."""
+    probe = min(nb_max, 20000)
+    tf, ts = oracle_run(oracle_data(probe, lo, hi, dt), nthreads)
+    rate = probe / max(tf + ts, 1e-6)
+    return int(max(min(nb_max, rate * seconds), min(nb_max, 1000)))
+
+
+def oracle_baseline(nb: int, lo: int, hi: int, dt, budget_s: float):
+    """cpu_baseline: the oracle as it stands on the host cores, on a bounded
+    sample (the workload's first blocks), all cores (OpenMP over blocks) and
+    one thread; GETRF and GETRS timed separately; median of 3."""
+    import oracle
+    cores = oracle.max_threads()
+    n_all = oracle_sample_size(nb, lo, hi, dt, budget_s / 5.0)
+    data = oracle_data(n_all, lo, hi, dt)
+    reps = [oracle_run(data) for _ in range(3)]
+    tf = float(np.median([r[0] for r in reps]))
+    ts = float(np.median([r[1] for r in reps]))
+    n_one = min(n_all, max(1000, int(n_all / max(cores, 1) / 2)))
+    one = oracle_run((data[0][:n_one], data[1][:n_one + 1], data[2][:n_one + 1], data[3], data[4]), 1)
+    getrf_b, getrs_b = algorithmic_bytes(data[0], dt)
+    return {"value": n_all / (tf + ts), "unit": "blocks/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {n_all} blocks of the workload (GETRF+GETRS, OpenMP over blocks, median of 3)",
+            "cpu_model": cpu_model(), "getrf_s": tf, "getrs_s": ts,
+            "gbs": (getrf_b + getrs_b) / (tf + ts) / 1e9,
+            "single_thread": {"value": n_one / (one[0] + one[1]), "unit": "blocks/s",
+                              "sample": f"first {n_one} blocks", "getrf_s": one[0], "getrs_s": one[1]}}
 
 
 def run_reference(args, ws, rank):
-    nb, lo, hi, dt, desc = CONFIGS[args.config]
+    """Reference arm of this tier: the CPU oracle as it stands, timed on the
+    host cores, on the same workload / metric as our arm.  Each step is one
+    GETRF + GETRS pass over a bounded sample (the workload's first blocks,
+    sized so the whole run ends within a few minutes)."""
+    nb_total, lo, hi, dt, desc, scaling = workload(args, ws)
     if rank != 0:
         return
-    budget = max(2.0, min(20.0, 60.0 / max(args.steps + args.warmup, 1)))
+    per_step = max(0.3, min(2.0, 90.0 / max(args.steps + args.warmup, 1)))
+    n = oracle_sample_size(nb_total, lo, hi, dt, per_step)
+    data = oracle_data(n, lo, hi, dt)
+    import oracle
+    cores = oracle.max_threads()
     times = []
-    blocks = 0
     for i in range(args.warmup + args.steps):
-        done, t, cores = oracle_sample(nb, lo, hi, dt, budget)
+        tf, ts = oracle_run(data)
         if i >= args.warmup:
-            times.append(t)
-            blocks += done
+            times.append(tf + ts)
     tot = sum(times)
-    value = blocks / tot
+    value = n * len(times) / tot
     line = {
-        "impl": "reference", "metric": "blocks/s (batched LU + solve)", "value": value, "unit": "blocks/s",
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "blocks/s",
         "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * tot / max(args.steps, 1), "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": 1e3 * tot / max(args.steps, 1), "higher_is_better": True, "scaling": scaling,
         "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32", "data": "synthetic",
-        "config": {"workload": desc, "sample": f"first {blocks // max(args.steps, 1)} blocks of the workload per step"},
+        "config": {"workload": desc, "nblocks_total": nb_total,
+                   "sample": f"each step: GETRF+GETRS over the first {n} blocks of the workload"},
         "cpu_baseline": {"value": value, "unit": "blocks/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{blocks // max(args.steps, 1)} blocks per step (GETRF+GETRS)"},
+                         "sample": f"{n} blocks per step (GETRF+GETRS, OpenMP over blocks)",
+                         "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "blocks/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -211,10 +280,7 @@ def run_reference(args, ws, rank):
 # --------------------------------------------------------------------------
 def run_ours(args, ws, rank, local):
     from paper_conf_icpp_anztdfq17_b200 import bj
-    nb_per, lo, hi, dt, desc = CONFIGS[args.config]
-    if args.nblocks:
-        nb_per = args.nblocks
-    nb_total = nb_per * ws
+    nb_total, lo, hi, dt, desc, scaling = workload(args, ws)
     # --- partition (row a6): global sizes from the counter generator
     from paper_conf_icpp_anztdfq17_b200 import dist as D
     sizes_all = bj.synth_sizes(nb_total, lo, hi)
@@ -307,6 +373,8 @@ def run_ours(args, ws, rank, local):
     t_ms = max_over_ranks(t_total_ms, ws)
     per = np.array(per)
     plan_ms, getrf_ms, getrs_ms = (float(per[:, j].mean()) for j in range(3))
+    step_each = per.sum(axis=1)
+    step_med, step_min = float(np.median(step_each)), float(step_each.min())
     getrf_ms = max_over_ranks(getrf_ms, ws)
     getrs_ms = max_over_ranks(getrs_ms, ws)
     clocks = sampler.summary()
@@ -356,18 +424,17 @@ def run_ours(args, ws, rank, local):
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:
-        done_b, t_cpu, cores = oracle_sample(nb_per, lo, hi, dt, args.cpu_budget)
-        cpu = {"value": done_b / t_cpu, "unit": "blocks/s", "cores": cores, "kind": "oracle",
-               "sample": f"first {done_b} blocks of the workload (GETRF+GETRS, OpenMP over blocks)"}
+        cpu = oracle_baseline(nb_total, lo, hi, dt, args.cpu_budget)
 
     if rank == 0:
         line = {
-            "metric": "blocks/s (batched LU + solve)", "value": value, "unit": "blocks/s", "n_gpus": ws,
+            "metric": METRIC, "value": value, "unit": "blocks/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32",
+            "scaling": scaling, "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32",
             "data": "synthetic (counter-based splitmix64, generated on device)",
-            "config": {"workload": desc, "nblocks_total": nb_total, "sizes": f"U{{{lo}..{hi}}}",
-                       "step": "layout + plan + getrf + getrs", "parallelism": f"dp{ws} (contiguous cost-balanced shards)",
+            "config": {"workload": desc, "nblocks_total": nb_total, "nblocks_rank0": nb, "sizes": f"U{{{lo}..{hi}}}",
+                       "step": "layout + plan + getrf + getrs",
+                       "parallelism": f"dp{ws} (contiguous cost-balanced shards, {scaling} scaling)",
                        "l2": f"inputs larger than L2: each step factors its own pristine {copy_bytes / 1e9:.2f} GB copy"},
             "roofline": {"bound": "hbm", "kernel": f"bj_{dom}_vbatched (size-class launches)", "achieved": achieved,
                          "peak": hbm, "unit": "GB/s", "frac": achieved / hbm, "traffic": traffic,
@@ -375,6 +442,7 @@ def run_ours(args, ws, rank, local):
             "step_hbm": {"algorithmic_bytes": step_bytes, "achieved_gbs": step_bytes / (ms_per_step * 1e-3) / 1e9,
                          "frac": step_bytes / (ms_per_step * 1e-3) / 1e9 / hbm},
             "breakdown_ms": {"layout_plan": plan_ms, "getrf": getrf_ms, "getrs": getrs_ms},
+            "step_ms_rank0": {"median": step_med, "min": step_min},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
             "nonzero_info_blocks": bad,
         }
@@ -490,6 +558,22 @@ def run_fem(args, ws, rank, local):
         print(json.dumps(line), flush=True)
 
 
+def spawn(n: int) -> int:
+    """`bench.py --gpus N` started as a plain process: re-launch it under
+    torch.distributed.run with one rank per GPU (the launch the driver uses)."""
+    import socket
+    import subprocess
+    if torch.cuda.device_count() < n:
+        print(json.dumps({"error": f"--gpus {n} requested but {torch.cuda.device_count()} GPU(s) visible"}))
+        return 2
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -502,8 +586,12 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="multi-GPU batched configs: shard the config's batch (strong) or replicate it per GPU (weak)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 0)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn(args.gpus))
     if args.impl == "reference":
         # the CPU oracle arm: rank 0 alone runs it; other ranks exit without work
         ws = int(os.environ.get("WORLD_SIZE", "1"))

@@ -262,3 +262,93 @@ def uniform_block_ptr(n: int, b: int, r0: int = 0) -> np.ndarray:
     """Blocks of b consecutive rows over rows [0, n) (last block n mod b)."""
     edges = list(range(0, n, b)) + [n]
     return np.asarray(edges, dtype=np.int32)
+
+
+# --------------------------------------------------------------------------
+# C implementation of the same generators (bj_synth/fastgen.c) for full-size
+# inputs; checked bit for bit against the numpy functions above
+# (tests/test_synth.py).
+# --------------------------------------------------------------------------
+import ctypes as _ct
+import os as _os
+import subprocess as _sp
+
+_HERE = _os.path.dirname(_os.path.abspath(__file__))
+_FAST_SRC = _os.path.join(_HERE, "fastgen.c")
+_FAST_LIB = _os.path.join(_HERE, "libbjs_fast.so")
+_fast = None
+
+
+def build_fast(force: bool = False) -> str:
+    if force or not _os.path.exists(_FAST_LIB) or _os.path.getmtime(_FAST_LIB) < _os.path.getmtime(_FAST_SRC):
+        tmp = _FAST_LIB + ".tmp%d" % _os.getpid()
+        _sp.check_call(["gcc", "-std=gnu99", "-O2", "-fopenmp", "-fPIC", "-shared", "-Wall", _FAST_SRC,
+                        "-o", tmp, "-lm"])
+        _os.replace(tmp, _FAST_LIB)
+    return _FAST_LIB
+
+
+def _fastlib():
+    global _fast
+    if _fast is None:
+        build_fast()
+        L = _ct.CDLL(_FAST_LIB)
+        P, I64, I32 = _ct.c_void_p, _ct.c_int64, _ct.c_int
+        for s in ("d", "s"):
+            getattr(L, f"bjs_block_values_{s}").argtypes = [I64, I64, I32, P, P, P, P]
+            getattr(L, f"bjs_rhs_values_{s}").argtypes = [I64, I64, P, P, P, P]
+            getattr(L, f"bjs_fem_fill_{s}").argtypes = [I32, I32, I32, I32, I64, I64, P, P, P]
+            getattr(L, f"bjs_fem_fill_{s}").restype = I32
+        L.bjs_fem_row_ptr.argtypes = [I32, I32, I32, I32, I64, I64, P]
+        L.bjs_fem_row_ptr.restype = I32
+        _fast = L
+    return _fast
+
+
+def _pp(a):
+    return None if a is None else a.ctypes.data_as(_ct.c_void_p)
+
+
+def _sfx(dtype):
+    return "d" if np.dtype(dtype) == np.float64 else "s"
+
+
+def block_values_fast(sizes, val_off, first: int = 0, dtype=np.float64, kind: str = "uniform", ids=None):
+    """Same output as block_values() (C, OpenMP)."""
+    sizes = np.ascontiguousarray(sizes, dtype=np.int32)
+    val_off = np.ascontiguousarray(val_off, dtype=np.int64)
+    nb = len(sizes)
+    out = np.empty(int(val_off[nb]), dtype=dtype)
+    idv = None if ids is None else np.ascontiguousarray(ids, dtype=np.int64)
+    getattr(_fastlib(), f"bjs_block_values_{_sfx(dtype)}")(nb, first, 0 if kind == "uniform" else 1, _pp(sizes),
+                                                          _pp(val_off), _pp(idv), _pp(out))
+    return out
+
+
+def rhs_values_fast(sizes, first: int = 0, dtype=np.float64, ids=None):
+    """Same output as rhs_values() (C, OpenMP)."""
+    sizes = np.ascontiguousarray(sizes, dtype=np.int32)
+    nb = len(sizes)
+    vec = np.zeros(nb + 1, dtype=np.int64)
+    np.cumsum(sizes, out=vec[1:])
+    out = np.empty(int(vec[nb]), dtype=dtype)
+    idv = None if ids is None else np.ascontiguousarray(ids, dtype=np.int64)
+    getattr(_fastlib(), f"bjs_rhs_values_{_sfx(dtype)}")(nb, first, _pp(sizes), _pp(vec), _pp(idv), _pp(out))
+    return out
+
+
+def fem_csr_fast(nx: int, ny: int, nz: int, r0: int = 0, r1: int | None = None, dtype=np.float64,
+                 skew: bool = True):
+    """Same output as FemGrid(nx, ny, nz, skew).csr(r0, r1, dtype) (C, OpenMP)."""
+    n = 3 * nx * ny * nz
+    r1 = n if r1 is None else r1
+    L = _fastlib()
+    rp = np.empty(r1 - r0 + 1, dtype=np.int64)
+    if L.bjs_fem_row_ptr(nx, ny, nz, int(skew), r0, r1, _pp(rp)) != 0:
+        raise ValueError("bad FEM row range")
+    nnz = int(rp[-1])
+    col = np.empty(nnz, dtype=np.int32)
+    val = np.empty(nnz, dtype=dtype)
+    if getattr(L, f"bjs_fem_fill_{_sfx(dtype)}")(nx, ny, nz, int(skew), r0, r1, _pp(rp), _pp(col), _pp(val)) != 0:
+        raise ValueError("bad FEM row range")
+    return rp, col, val

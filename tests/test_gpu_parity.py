@@ -222,47 +222,84 @@ def test_gesv_host_end_to_end():
     assert np.array_equal(bits(x_h.numpy()), bits(x_o))
 
 
-@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_c3_full_size_sampled(dtype):
-    """Config C3 at full size (1M blocks, m ~ U{4..32}) in the launch
-    configuration bench.py times; 3,000 sampled blocks recomputed one by one by
-    the oracle from the host generator."""
-    nb = 1_000_000
-    sizes_d = bj.synth_sizes(nb, 4, 32)
+def _c3_device(nb, dtype, first=0):
+    """C3-shaped batch generated on the device (the bench's inputs), factored
+    and solved in the bench's launch configuration (plan reused)."""
+    sizes_d = bj.synth_sizes(nb, 4, 32, first=first)
     batch = bj.new_batch(sizes_d, dtype)
-    bj.synth_blocks(batch)
-    b = bj.synth_rhs(batch)
+    bj.synth_blocks(batch, first=first)
+    b = bj.synth_rhs(batch, first=first)
     plan = bj.Plan(batch.sizes)
     nvec = int(batch.vec_off[-1].item())
-    piv = torch.empty(nvec, dtype=torch.int32, device="cuda")
-    info = torch.empty(nb, dtype=torch.int32, device="cuda")
+    piv = torch.empty(max(nvec, 1), dtype=torch.int32, device="cuda")
+    info = torch.empty(max(nb, 1), dtype=torch.int32, device="cuda")
     x = torch.empty_like(b)
     bj.getrf(batch, piv, info, plan=plan)
     bj.getrs(batch, piv, b, x, plan=plan)
+    plan.close()
+    return batch, piv[:nvec], info[:nb], x[:nvec]
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_c3_full_size_all_blocks(dtype):
+    """Config C3 at full size (1M blocks, m ~ U{4..32}) in the launch
+    configuration bench.py times, EVERY block compared with the oracle:
+    pivots, info, L\\U bits and x bits.  The oracle's input comes from the host
+    generator (bj_synth, C implementation), never from the device."""
+    nb = 1_000_000
+    batch, piv, info, x = _c3_device(nb, dtype)
     torch.cuda.synchronize()
-    assert int((info != 0).sum().item()) == 0
     sizes = S.block_sizes(nb, 4, 32)
-    assert np.array_equal(sizes_d.cpu().numpy(), sizes)
-    rng = np.random.default_rng(77)
-    ids = np.unique(np.concatenate([rng.choice(nb, 2998, replace=False), [0, nb - 1]]))
-    vo = batch.val_off.cpu().numpy()
-    ve = batch.vec_off.cpu().numpy()
-    vec_h, val_h = host_layout(sizes, dtype)
-    assert np.array_equal(vo, val_h) and np.array_equal(ve, vec_h)
-    LU_all = batch.values
+    vec, val = host_layout(sizes, dtype)
+    assert np.array_equal(batch.sizes.cpu().numpy(), sizes)
+    assert np.array_equal(batch.vec_off.cpu().numpy(), vec) and np.array_equal(batch.val_off.cpu().numpy(), val)
+    A = S.block_values_fast(sizes, val, dtype=NP[dtype])
+    b = S.rhs_values_fast(sizes, dtype=NP[dtype])
+    LU_o, piv_o, info_o = oracle.getrf_batch(sizes, val, vec, A)
+    x_o = oracle.getrs_batch(sizes, val, vec, LU_o, piv_o, b)
+    assert np.array_equal(info.cpu().numpy(), info_o)
+    assert int((info_o != 0).sum()) == 0
+    assert np.array_equal(piv.cpu().numpy(), piv_o)
+    LU_d = batch.values.cpu().numpy()[: len(LU_o)]
+    diff = np.flatnonzero(bits(LU_d) != bits(LU_o))
+    assert diff.size == 0, f"{diff.size} L\\U elements differ, first at {diff[:5]}"
+    assert np.array_equal(bits(x.cpu().numpy()), bits(x_o))
+    # backward error on a sample (the bits are already the oracle's)
+    ids = np.arange(0, nb, 997)
     ss = sizes[ids]
     svec, sval = host_layout(ss, dtype)
-    A_s = S.block_values(ss, sval, dtype=NP[dtype], ids=ids)
-    b_s = S.rhs_values(ss, dtype=NP[dtype], ids=ids)
-    LU_o, piv_o, info_o = oracle.getrf_batch(ss, sval, svec, A_s)
-    x_o = oracle.getrs_batch(ss, sval, svec, LU_o, piv_o, b_s)
-    lu_idx = np.concatenate([np.arange(vo[i], vo[i] + sizes[i] ** 2) for i in ids])
-    v_idx = np.concatenate([np.arange(ve[i], ve[i] + sizes[i]) for i in ids])
-    LU_d = LU_all[torch.from_numpy(lu_idx).cuda()].cpu().numpy()
-    piv_d = piv[torch.from_numpy(v_idx).cuda()].cpu().numpy()
-    x_d = x[torch.from_numpy(v_idx).cuda()].cpu().numpy()
-    LU_o_packed = np.concatenate([LU_o[sval[j]: sval[j] + ss[j] ** 2] for j in range(len(ids))])
-    assert np.array_equal(piv_d, piv_o)
-    assert np.array_equal(bits(LU_d), bits(LU_o_packed))
-    assert np.array_equal(bits(x_d), bits(x_o))
-    assert backward_error(ss, sval, svec, A_s, b_s, x_o) <= TOL[dtype]
+    A_s = S.block_values_fast(ss, sval, dtype=NP[dtype], ids=ids)
+    b_s = S.rhs_values_fast(ss, dtype=NP[dtype], ids=ids)
+    x_s = np.concatenate([x_o[vec[i]: vec[i] + sizes[i]] for i in ids])
+    assert backward_error(ss, sval, svec, A_s, b_s, x_s) <= TOL[dtype]
+
+
+@pytest.mark.parametrize("G", [2, 4, 8])
+def test_c3_logical_sharding(G):
+    """Hot-path row a6 on one device: the C3 batch (1M blocks) split into G
+    contiguous cost-balanced shards (bj_partition), each regenerated from the
+    counter generator with first= and factored/solved on its own; the
+    concatenated pivots, info, L\\U and x are bit-equal to the unsharded run
+    (which test_c3_full_size_all_blocks ties to the oracle block by block)."""
+    nb = 1_000_000
+    dtype = torch.float64
+    full, piv, info, x = _c3_device(nb, dtype)
+    sizes = S.block_sizes(nb, 4, 32)
+    bounds = bj.partition(sizes, G)
+    assert np.array_equal(bounds, oracle.partition(sizes, G))
+    assert bounds[0] == 0 and bounds[-1] == nb and np.all(np.diff(bounds) > 0)
+    cost = np.add.reduceat(sizes.astype(np.int64) ** 2, bounds[:-1])
+    assert cost.max() / cost.mean() < 1.001                  # balanced by m^2
+    vo = full.val_off.cpu().numpy()
+    ve = full.vec_off.cpu().numpy()
+    for r in range(G):
+        s, e = int(bounds[r]), int(bounds[r + 1])
+        sb, sp, si, sx = _c3_device(e - s, dtype, first=s)
+        assert torch.equal(sb.sizes, full.sizes[s:e])
+        assert torch.equal(si, info[s:e])
+        assert torch.equal(sp, piv[ve[s]: ve[e]])
+        n = int(vo[e] - vo[s])
+        assert torch.equal(sb.values[:n].view(torch.int64), full.values[vo[s]: vo[e]].view(torch.int64))
+        assert torch.equal(sx.view(torch.int64), x[ve[s]: ve[e]].view(torch.int64))
+        del sb, sp, si, sx
+    torch.cuda.synchronize()

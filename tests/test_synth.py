@@ -76,3 +76,41 @@ def test_hub_tail_is_pareto_like():
     assert ks.min() >= 100
     # Pareto(1.5, 100): median 100 * 2^(2/3) = 158.7
     assert 120 < np.median(ks) < 200
+
+
+def test_fast_generator_matches_numpy():
+    """bj_synth/fastgen.c reproduces the numpy generators bit for bit."""
+    sizes = S.block_sizes(3000, 1, 32, first=777)
+    for dt, es in ((np.float64, 8), (np.float32, 4)):
+        vec, val = S.packed_offsets(sizes, es)
+        for kind in ("uniform", "int"):
+            a = S.block_values(sizes, val, first=777, dtype=dt, kind=kind)
+            b = S.block_values_fast(sizes, val, first=777, dtype=dt, kind=kind)
+            assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+        ids = np.arange(5000, 8000, dtype=np.int64)[::-1].copy()
+        a = S.block_values(sizes, val, dtype=dt, ids=ids)
+        b = S.block_values_fast(sizes, val, dtype=dt, ids=ids)
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+        a = S.rhs_values(sizes, first=777, dtype=dt)
+        b = S.rhs_values_fast(sizes, first=777, dtype=dt)
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8))
+
+
+def test_fast_fem_matches_numpy():
+    g = S.FemGrid(9, 8, 7)            # W > 0: hub rows possible
+    n = g.n
+    for dt in (np.float64, np.float32):
+        for r0, r1 in ((0, n), (100, 700)):
+            rp, col, val = g.csr(r0, r1, dtype=dt)
+            rp2, col2, val2 = S.fem_csr_fast(9, 8, 7, r0, r1, dtype=dt)
+            assert np.array_equal(rp, rp2) and np.array_equal(col, col2)
+            assert np.array_equal(val.view(np.uint8), val2.view(np.uint8))
+    # a grid big enough to contain hub rows (0.1 % of rows)
+    g = S.FemGrid(30, 30, 12)
+    hubs = [r for r in range(g.n) if g.n_extra(r) > 0][:3]
+    assert hubs, "expected hub rows"
+    for r in hubs:
+        rp, col, val = g.csr(r, r + 2)
+        rp2, col2, val2 = S.fem_csr_fast(30, 30, 12, r, r + 2)
+        assert np.array_equal(rp, rp2) and np.array_equal(col, col2)
+        assert np.array_equal(val.view(np.uint8), val2.view(np.uint8))
