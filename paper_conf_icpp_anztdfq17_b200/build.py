@@ -36,7 +36,8 @@ def _jobs():
         jobs.append((src, [], src.replace(".cu", ".o")))
     for kind in ("getrf", "getrs"):
         for dt in DTYPES:
-            for lo, hi in CLASSES:
+            classes = CLASSES if kind == "getrs" else CLASSES[:3] + [(m, m) for m in range(17, 33)]
+            for lo, hi in classes:
                 jobs.append((f"{kind}_inst.cu", [f"-DBJ_R={dt}", f"-DBJ_LO={lo}", f"-DBJ_HI={hi}"],
                              f"{kind}_{dt[0]}_{lo}_{hi}.o"))
     return jobs

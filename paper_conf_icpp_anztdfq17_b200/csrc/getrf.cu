@@ -1,4 +1,4 @@
-// getrf.cu -- host driver of hot-path row a3 (kernels: getrf_kernels.cuh,
+// getrf.cu -- host driver of hot-path row a3 (kernels: getrf_fast.cuh,
 // instantiated per (dtype, size class) in getrf_inst.cu so they compile in
 // parallel).
 #include "getrf_fast.cuh"
@@ -27,11 +27,25 @@ bj_status getrf_run(R *A, const int64_t *val_off, const int64_t *vec_off, int32_
     if (p.nblocks == 0) return BJ_OK;
     char *scratch = nullptr;
     BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch, 16 + sizeof(int32_t) * (size_t)p.nblocks, s));
+    // the scratch is released (stream-ordered) on every return path
+    struct Free {
+        char *p;
+        cudaStream_t s;
+        ~Free() { cudaFreeAsync(p, s); }
+    } guard{scratch, s};
     unsigned *safe_count = reinterpret_cast<unsigned *>(scratch);
     int32_t *safe_list = reinterpret_cast<int32_t *>(scratch + 16);
     BJ_CUDA_TRY(cudaMemsetAsync(safe_count, 0, sizeof(unsigned), s));
     bj_status st;
-    if ((st = launch_getrf_fast<R, 17, 32>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    // orders 32..17: one kernel per order (each gets the register allocation of
+    // its own order; chained by programmatic dependent launch), then the
+    // sub-warp classes.
+#define BJ_GETRF_M(M) \
+    if ((st = launch_getrf_fast<R, M, M>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
+    BJ_GETRF_M(32) BJ_GETRF_M(31) BJ_GETRF_M(30) BJ_GETRF_M(29) BJ_GETRF_M(28) BJ_GETRF_M(27) BJ_GETRF_M(26)
+    BJ_GETRF_M(25) BJ_GETRF_M(24) BJ_GETRF_M(23) BJ_GETRF_M(22) BJ_GETRF_M(21) BJ_GETRF_M(20) BJ_GETRF_M(19)
+    BJ_GETRF_M(18) BJ_GETRF_M(17)
+#undef BJ_GETRF_M
     if ((st = launch_getrf_fast<R, 9, 16>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
     if ((st = launch_getrf_fast<R, 5, 8>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
     if ((st = launch_getrf_fast<R, 1, 4>(A, val_off, vec_off, piv, info, p, safe_list, safe_count, s)) != BJ_OK) return st;
@@ -39,7 +53,6 @@ bj_status getrf_run(R *A, const int64_t *val_off, const int64_t *vec_off, int32_
     BJ_LAUNCH_CHECK();
     k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
     BJ_LAUNCH_CHECK();
-    BJ_CUDA_TRY(cudaFreeAsync(scratch, s));
     return BJ_OK;
 }
 

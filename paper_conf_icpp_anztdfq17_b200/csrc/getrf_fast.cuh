@@ -1,41 +1,51 @@
 #pragma once
 // getrf_fast.cuh -- hot-path row a3: variable-size batched LU with implicit
 // (swap-free) partial pivoting, Fig. 1 bottom, section III.A
-// (P:400-464).  Production kernels (the earlier variants in getrf_kernels.cuh
-// are kept for the micro benchmarks).
+// (P:400-464).
 //
 // Design, driven by B200 measurements
-// (scripts/micro/*.cu, profiles/):
+// (scripts/micro/prims.cu -> profiles/r02/micro_prims.txt):
 //  * blocks grouped by exact order m (plan, layout.cu); one persistent kernel
 //    per size class {1-4, 5-8, 9-16, 17-32}; a warp takes a "task" of
 //    G = 32/T same-order blocks, a block occupies a tile of T = pow2ceil(m)
 //    lanes and lane r holds row r in registers (static indices: the code is
 //    fully unrolled per m).  A is read from HBM once and no lane
-//    computes on the reference's 32 x 32 padding.
-//  * The per-step critical path is the dependent chain pivot search ->
-//    pivot broadcast -> division -> update of column k+1 -> next search.
-//    Measured on B200 (one warp alone) it was ~400 cycles per step with
-//    REDUX + 2 VOTEs + a shared-memory round trip + the full division; here:
-//      - one REDUX.MAX per tile on a key that packs the candidate flag, the
-//        top 26 bits of |a| and the inverted lane, so the max also names the
-//        pivot lane; an ambiguity VOTE (another candidate with the same
-//        truncated key) runs off the critical path and triggers an exact
-//        pass only in that rare case -> exactly the oracle's order and tie
-//        rule (R1, R2);
-//      - every lane refines 1/a_kk of its own candidate while the search
-//        runs; the pivot's reciprocal is broadcast with the pivot, leaving a
-//        3-operation IEEE quotient (Num::div_pre_u, bit-identical to
-//        __ddiv_rn) on the chain;
-//      - full-warp tiles broadcast by SHFL from the warp-uniform pivot lane
-//        (cheap path of the shuffle unit, ~0.5 SM cycle per 32-bit word);
-//        sub-warp tiles publish through a per-warp smem slot / row buffer.
-//  * The GER is branch-free: rows that must not change (pivoted rows, padding
-//    lanes, singular steps R4) get the multiplier +0 and fma(-0, u, a) == a
-//    bit for bit whenever u is finite and a != -0.  That holds at every step
-//    if the block's entries are finite, not -0 and below 2^990 (no new -0 can
-//    arise and partial pivoting grows entries by at most 2^31 in 32 steps).
-//    Blocks failing that check at load time are deferred to a list and
-//    factored by k_getrf_safe (plain predicated algorithm in smem).
+//    computes on the reference's 32 x 32 padding.  The next
+//    task's blocks are staged into shared memory by the bulk-copy (TMA)
+//    engine while the current task is factored.
+//  * Step k (Fig. 1 bottom lines 5-15):
+//      - pivot search: one REDUX.MAX per tile on a key that packs the
+//        candidate flag, the top 26 bits of |a| and the inverted lane, so the
+//        max also names the pivot lane with the lowest-row tie rule (R1, R2).
+//        A candidate whose exact |a| exceeds the chosen pivot's (possible
+//        only when two values agree in those 26 bits) sets a per-tile redo
+//        flag; the tile is then factored again by k_getrf_safe with exact
+//        64-bit keys.  Exact ties are resolved by the lane order directly.
+//      - broadcast of the pivot row: full-warp tiles (m = 17..32) use SHFL
+//        from the warp-uniform pivot lane -- 0.27 SM-cycles per 32-bit word,
+//        against 4.2 SM-cycles for a one-lane STS.128 plus 1.2 for the
+//        LDS.128 broadcast (measured, micro_prims.txt); sub-warp tiles have a
+//        different pivot lane per tile (SHFL at 1.0 SM-cycle per word), so
+//        they publish through a per-warp shared-memory row buffer.
+//      - SCAL: every candidate refines 1/a_kk of its own entry while the
+//        search runs (full-warp tiles); the pivot's reciprocal travels with
+//        the pivot, leaving the 3-operation IEEE quotient (Num::div_pre_flag,
+//        bit-identical to __ddiv_rn / __fdiv_rn) on the critical path.
+//      - GER: branch-free, one FMA per element: rows that must not change
+//        (pivoted rows, padding lanes, singular steps R4) use the multiplier
+//        +0, and fma(-0, u, a) == a bit for bit unless a == -0 (nvcc turns a
+//        predicated DFMA into DFMA + 2 FSEL, 5 instead of 3 issue slots per
+//        element).  No -0 can reach a frozen row: inputs hold none, SCAL
+//        writes only column k (never touched again) and a GER result is -0
+//        only through underflow.  Underflow is excluded by magnitudes: if
+//        every input and every final L\U entry is 0 or in [2^-450, 2^990)
+//        (fp32: [2^-39, 2^96)), every product l*u is 0 or >= 2^-900, a
+//        result below it in magnitude cannot cancel further, and every
+//        nonzero intermediate stays >= 2^-1006 (fp32 2^-126), above the
+//        subnormal range.  Blocks failing the input test go to k_getrf_safe
+//        at load time, blocks failing the output test are redone by it.
+//  * Partial pivoting grows entries by at most 2^31 in 32 steps, so every
+//    fast-path intermediate is finite.
 //  * Combined row swap at write-back: lane r stores its row at
 //    position tag-1 of every column and perm[tag-1] = r.
 #include "common.cuh"
@@ -44,19 +54,18 @@
 namespace bj {
 
 constexpr int kFastThreads = 128;
-#ifdef BJ_TRACE
-__device__ long long g_ftrace[64];
-#endif
 
-// "Safe for the zero-multiplier GER" (see header comment).
-template <typename R> __device__ __forceinline__ bool zero_mult_safe(R x);
-template <> __device__ __forceinline__ bool zero_mult_safe<double>(double x) {
+// Entries the fast path accepts, on input and in the final L\U (header
+// comment): +0, or |x| in [2^-450, 2^990) (fp32 [2^-39, 2^96)).  -0 and
+// non-finite values fail.
+template <typename R> __device__ __forceinline__ bool fast_ok(R x);
+template <> __device__ __forceinline__ bool fast_ok<double>(double x) {
     const unsigned hi = (unsigned)__double2hiint(x), lo = (unsigned)__double2loint(x);
-    return ((hi & 0x7fffffffu) < 0x7DD00000u) && !(hi == 0x80000000u && lo == 0u);
+    return ((hi & 0x7fffffffu) - 0x23D00000u < 0x7DD00000u - 0x23D00000u) || ((hi | lo) == 0u);
 }
-template <> __device__ __forceinline__ bool zero_mult_safe<float>(float x) {
+template <> __device__ __forceinline__ bool fast_ok<float>(float x) {
     const unsigned b = __float_as_uint(x);
-    return ((b & 0x7fffffffu) < (221u << 23)) && b != 0x80000000u;
+    return ((b & 0x7fffffffu) - (88u << 23) < (223u << 23) - (88u << 23)) || b == 0u;
 }
 
 // Per-tile max of a 32-bit key.  Full warp: one REDUX; 2 or 4 tiles: one
@@ -81,23 +90,49 @@ __device__ __forceinline__ unsigned tile_max_key(unsigned key, int t) {
     }
 }
 
+// Row stride of the panel buffer: fp64 34 elements (272 B = 17 x 16 B, an
+// odd number of 16-B units, so the STS.128 of the panel's pivot lanes hit
+// distinct bank groups)
+// (fp32: 36 elements = 144 B = 9 x 16 B).
+template <typename R> __host__ __device__ constexpr int panel_stride() { return sizeof(R) == 8 ? 34 : 36; }
+constexpr int kMaxPanel = 4;
 template <typename R>
 struct FastSmem {
-    R slot[64];     // per lane: (a_kk, refined 1/a_kk) -- sub-warp tiles
-    R row[2][32];   // pivot-row buffers (alternating steps), T elements per tile
+    R row[32];                                    // pivot-row buffer, T elements per tile (sub-warp tiles)
+    R panel[kMaxPanel][panel_stride<R>()];        // full-warp tiles: the panel's pivot rows (stale trailing part)
 };
 
-// Compile-time options (defaults chosen by scripts/micro/getrf_bench.cu on the
-// C3 order mix): kFastShflW32 -- full-warp tiles broadcast by SHFL instead of
-// smem; kFastPreRcp -- every lane pre-refines 1/a_kk (shorter chain, more
-// instructions).
-constexpr int kFastShflW32 = 1, kFastPreRcp = 2, kFastHybrid = 4, kFastDblBuf = 8;
-// Micro-benchmark-only ablations (wrong results; scripts/micro/getrf_bench.cu):
-// skip the pivot-row publish / the division / the pivot search.
-constexpr int kFastXNoPub = 16, kFastXNoDiv = 32, kFastXNoSearch = 64, kFastXAllLanes = 128, kFastXOnePair = 256;
+// Compile-time variants (scripts/micro/getrf_var.cu measures them):
+//   kPre  -- every candidate refines 1/a_kk before the search (shorter chain,
+//            more instructions); otherwise 1/d is refined after the broadcast.
+//   kMin3 -- 3 CTAs (12 warps) per SM, 168 registers, instead of 4 (16 warps,
+//            128 registers).
+//   kVol  -- GER broadcast + FMA as volatile inline PTX (ptxas then keeps two
+//            SHFL pairs in flight instead of one).
+//   kPanel2/3/4 -- full-warp tiles: W-step panels (see getrf_w32_steps).
+//   kMin5 / kMin6 -- 5 / 6 CTAs (20 / 24 warps) per SM (102 / 85 registers).
+//   kMin4 -- 4 CTAs (16 warps) per SM (128 registers).
+constexpr int kPre = 1, kMin3 = 2, kVol = 4, kPanel2 = 8, kPanel3 = 16, kPanel4 = 32, kMin5 = 64, kMin6 = 128,
+              kMin4 = 256;
+__host__ __device__ constexpr int panel_width(int F) {
+    return (F & kPanel4) ? 4 : (F & kPanel3) ? 3 : (F & kPanel2) ? 2 : 1;
+}
 #ifndef BJ_FAST_DEFAULT
-#define BJ_FAST_DEFAULT 0
+#define BJ_FAST_DEFAULT 8
 #endif
+// Resident CTAs (of 4 warps) per SM: explicit flags, else by the registers
+// the largest order of the class needs (row in registers + ~50).
+template <typename R>
+__host__ __device__ constexpr int fast_min_blocks(int F, int MHI) {
+    return (F & kMin3) ? 3 : (F & kMin4) ? 4 : (F & kMin6) ? 6 : (F & kMin5) ? 5
+         : (MHI * (int)sizeof(R) / 4 <= 44) ? 6 : (MHI * (int)sizeof(R) / 4 <= 52) ? 5 : 4;
+}
+// Staging buffer per warp: one task = 32/T blocks of order <= MHI.
+template <typename R>
+__host__ __device__ constexpr int stage_elems(int MLO, int MHI) {
+    return MLO >= 17 ? (MHI * MHI + 16 / (int)sizeof(R) - 1) / (16 / (int)sizeof(R)) * (16 / (int)sizeof(R))
+                     : 32 * 32;
+}
 
 // Staging-buffer stride per tile: T*T elements rounded up to 16 bytes (the
 // bulk copy needs 16-B aligned destinations); 32/T tiles fit in 1024 elements.
@@ -116,20 +151,156 @@ struct FTask {
     int64_t vo;       // vec_off[blk]
 };
 
+// Broadcast of the pivot's value x to every lane of a full-warp tile.
+template <typename R>
+__device__ __forceinline__ R bcast(R x, int src) { return __shfl_sync(kFull, x, src); }
+__device__ __forceinline__ double vbcast(double x, int src) {
+    unsigned lo = __double2loint(x), hi = __double2hiint(x), rlo, rhi;
+    asm volatile("shfl.sync.idx.b32 %0, %1, %2, 0x1f, -1;" : "=r"(rlo) : "r"(lo), "r"(src));
+    asm volatile("shfl.sync.idx.b32 %0, %1, %2, 0x1f, -1;" : "=r"(rhi) : "r"(hi), "r"(src));
+    return __hiloint2double(rhi, rlo);
+}
+__device__ __forceinline__ float vbcast(float x, int src) {
+    float r;
+    asm volatile("shfl.sync.idx.b32 %0, %1, %2, 0x1f, -1;" : "=f"(r) : "f"(x), "r"(src));
+    return r;
+}
+__device__ __forceinline__ double vfma(double a, double b, double c) {
+    double d;
+    asm volatile("fma.rn.f64 %0, %1, %2, %3;" : "=d"(d) : "d"(a), "d"(b), "d"(c));
+    return d;
+}
+__device__ __forceinline__ float vfma(float a, float b, float c) {
+    float d;
+    asm volatile("fma.rn.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+    return d;
+}
+
+// Steps of a full-warp tile (M = 17..32) in W-step panels.
+//
+// Every step needs the pivot row at every lane.  A one-lane STS.128 costs
+// 4.2 SM-cycles whatever the number of active lanes (4 quarter-warp passes,
+// micro_prims.txt), and SHFL-broadcast DFMA chains are latency-bound, so the
+// panel amortises the publish over W pivot rows:
+//   1. steps k0..k0+W-1 run on the panel columns only (pivot search, SCAL,
+//      and the GER of the columns inside the panel, broadcast by SHFL);
+//   2. the W pivot lanes store the trailing part of their rows -- untouched
+//      since the panel began -- with the SAME predicated STS.128
+//      instructions (one store stream for W rows);
+//   3. every lane rebuilds the pivot rows' current values from them,
+//      u_s = st_s - sum_{s'<s} l(p_s, k0+s') u_s'  (fma chain in ascending
+//      s', exactly the updates pivot row p_s received in steps k0..k0+s-1),
+//      and applies the W deferred updates to its own trailing columns in
+//      ascending k.
+// Every element therefore sees the oracle's operations in the oracle's
+// order (R5): the rebuilt u_s is bit-identical to the pivot lane's own value.
+// Rows that must not change use multiplier 0 (zero-multiplier argument,
+// header comment).  Column k0+W, the next panel's first pivot column, is
+// updated first.
+template <typename R, int M, int W, bool PRE>
+__device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, int &inf, bool &redo, bool row_ok, int r,
+                                                FastSmem<R> &sm) {
+    constexpr int PS = panel_stride<R>();
+    constexpr int V = 16 / (int)sizeof(R);                 // elements per 16-B store / load
+    const unsigned lanebits = 0x80000000u | (unsigned)(31 - r);
+    static_for<0, (M + W - 1) / W>([&](auto pc) {
+        constexpr int k0 = decltype(pc)::value * W;
+        constexpr int kend = (k0 + W < M) ? k0 + W : M;
+        constexpr int nw = kend - k0;
+        R lk[W];                                           // this lane's multipliers of the panel's steps
+        int ipv[W];                                        // the panel's pivot lanes (warp-uniform)
+        static_for<0, nw>([&](auto sc) {
+            constexpr int sidx = decltype(sc)::value;
+            constexpr int k = k0 + sidx;
+            const bool cand = (tag == 0);
+            // PRE: every lane refines 1/a_kk of its own entry while the search runs
+            R y = R(0);
+            if constexpr (PRE) y = Num<R>::rcp_refine(a[k]);
+            // Fig. 1 bottom lines 5-7: key = candidate flag | top 26 bits of |a| | inverted lane.
+            const unsigned key = cand ? ((Num<R>::key_hi(a[k]) & 0x7fffffe0u) | lanebits) : 0u;
+            const unsigned kmax = __reduce_max_sync(kFull, key);
+            const int ipiv = 31 - (int)(kmax & 31u);
+            const R d = bcast(a[k], ipiv);                      // line 12: the pivot
+            const R yd = PRE ? bcast(y, ipiv) : Num<R>::rcp_refine(d);
+            // a candidate strictly larger than the chosen pivot: the truncated key was ambiguous
+            redo = redo || (cand && (fabs(a[k]) > fabs(d)));
+            if ((r == ipiv) && row_ok) tag = k + 1;             // line 9
+            const bool sing = (d == R(0));                      // R4
+            const bool upd = (tag == 0) && !sing;
+            bool bad = false;
+            const R q = Num<R>::div_nz_flag(a[k], d, yd, bad);  // line 13 (SCAL)
+            redo = redo || (upd && bad);
+            const R l = upd ? q : R(0);
+            if (upd) a[k] = q;
+            if (sing && inf == 0) inf = k + 1;
+            lk[sidx] = l;
+            ipv[sidx] = ipiv;
+            static_for<k + 1, kend>([&](auto jc) {              // lines 14-15 inside the panel
+                constexpr int j = decltype(jc)::value;          // fma(l, -u, a) == fma(-l, u, a) bitwise
+                a[j] = Num<R>::fma(l, -bcast(a[j], ipiv), a[j]);
+            });
+        });
+        if constexpr (kend < M) {
+            // 2. the panel's pivot lanes publish their stale trailing parts
+            const int slot = tag - 1 - k0;
+            const bool pub = row_ok && slot >= 0 && slot < nw;
+            R *dst = sm.panel[pub ? slot : 0];
+            __syncwarp();                                      // the previous panel's loads are done
+            constexpr int j0 = kend & ~(V - 1);
+            static_for<0, (M - j0 + V - 1) / V>([&](auto vc) {
+                constexpr int j = j0 + V * decltype(vc)::value;
+                if constexpr (sizeof(R) == 8) {
+                    if constexpr (j + 1 < M) st_shared_pred(pub, dst + j, a[j], a[j + 1]);
+                    else st_shared_pred(pub, dst + j, a[j]);
+                } else {
+                    if constexpr (j + 3 < M) st_shared_pred(pub, dst + j, a[j], a[j + 1], a[j + 2], a[j + 3]);
+                    else {
+                        if constexpr (j + 1 < M) st_shared_pred(pub, dst + j, a[j], a[j + 1]);
+                        else st_shared_pred(pub, dst + j, a[j]);
+                        if constexpr (j + 2 < M) st_shared_pred(pub, dst + j + 2, a[j + 2]);
+                    }
+                }
+            });
+            // multipliers among the panel's pivot rows: Lp[s][s'] = l(p_s, k0+s')
+            R Lp[W][W];
+            static_for<1, nw>([&](auto sc) {
+                constexpr int sidx = decltype(sc)::value;
+                static_for<0, sidx>([&](auto tc) {
+                    constexpr int t = decltype(tc)::value;
+                    Lp[sidx][t] = bcast(lk[t], ipv[sidx]);
+                });
+            });
+            __syncwarp();
+            // 3. rebuild the pivot rows and apply the W deferred updates, column by column
+            static_for<kend, M>([&](auto jc) {
+                constexpr int j = decltype(jc)::value;
+                R u[W];
+                static_for<0, nw>([&](auto sc) {
+                    constexpr int sidx = decltype(sc)::value;
+                    R v = sm.panel[sidx][j];
+                    static_for<0, sidx>([&](auto tc) {
+                        constexpr int t = decltype(tc)::value;
+                        v = Num<R>::fma(Lp[sidx][t], -u[t], v);
+                    });
+                    u[sidx] = v;
+                    a[j] = Num<R>::fma(lk[sidx], -v, a[j]);
+                });
+            });
+        }
+    });
+}
+
 // S: this tile's block staged in shared memory by the bulk copy (column-major,
 // leading dimension M); `after_load` runs once the block is in registers
 // (it re-arms the warp's staging buffer with the next task).
 template <typename R, int M, int F, class AfterLoad>
 __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &tk, const R *S,
-                                                const int64_t *__restrict__ vec_off, int32_t *__restrict__ piv,
-                                                int32_t *__restrict__ info, int32_t *__restrict__ safe_list,
-                                                unsigned *__restrict__ safe_count, FastSmem<R> &sm,
-                                                AfterLoad &&after_load) {
+                                                int32_t *__restrict__ piv, int32_t *__restrict__ info,
+                                                int32_t *__restrict__ safe_list, unsigned *__restrict__ safe_count,
+                                                FastSmem<R> &sm, AfterLoad &&after_load) {
     constexpr int T = tile_width(M);
-    constexpr bool W32 = (T == 32) && ((F & kFastShflW32) != 0);
-    constexpr bool PRE = (F & kFastPreRcp) != 0;
-    constexpr bool HYB = (T == 32) && !W32 && ((F & kFastHybrid) != 0);
-    constexpr bool DBL = (F & kFastDblBuf) != 0;
+    constexpr bool W32 = (T == 32);
+    constexpr bool PRE = W32 && (F & kPre) != 0;
     const int lane = threadIdx.x & 31;
     const int t = lane / T;
     const int r = lane % T;
@@ -143,7 +314,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     static_for<0, M>([&](auto jc) {
         constexpr int j = decltype(jc)::value;
         a[j] = (tile_ok && r < M) ? S[r + j * M] : R(0);
-        ok = ok && zero_mult_safe(a[j]);
+        ok = ok && fast_ok(a[j]);
     });
     after_load();
     // Tiles with an entry outside the fast path's precondition go to the safe kernel.
@@ -156,74 +327,35 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     int tag = row_ok ? 0 : -1;      // 0: candidate; k+1: pivot of step k; -1: inactive lane
     int inf = 0;
     bool redo = false;              // pivot ambiguity or IEEE slow-path quotient in this tile
-    static_for<0, M>([&](auto kc) {
+    const unsigned lanebits = 0x80000000u | (unsigned)(31 - r);
+    if constexpr (W32 && panel_width(F) > 1) {
+        getrf_w32_steps<R, M, panel_width(F), (F & kPre) != 0>(a, tag, inf, redo, row_ok, r, sm);
+    } else static_for<0, M>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
-        // Alternating buffers: step k+1 publishes into the other buffer, so
-        // only the publish -> receive order needs a warp barrier (no barrier
-        // between this step's broadcast loads and the next step's stores).
-        R *buf = sm.row[DBL ? (k & 1) : 0] + tbase;
-#ifdef BJ_TRACE
-        if (blockIdx.x == 0 && threadIdx.x == 0) g_ftrace[k] = clock64();
-#endif
         const bool cand = (tag == 0);
-        // PRE: every lane refines 1/a_kk of its own candidate off the critical path.
         R y = R(0);
-        if constexpr (PRE) {
-            y = Num<R>::rcp_refine(a[k]);
-            if constexpr (!W32 && !HYB) {
-                if constexpr (sizeof(R) == 8) *reinterpret_cast<double2 *>(sm.slot + 2 * lane) = make_double2(a[k], y);
-                else *reinterpret_cast<float2 *>(sm.slot + 2 * lane) = make_float2(a[k], y);
-            }
-        }
+        if constexpr (PRE) y = Num<R>::rcp_refine(a[k]);
         // Fig. 1 bottom lines 5-7: key = candidate flag | top 26 bits of |a| | inverted lane.
-        const unsigned hi = Num<R>::key_hi(a[k]);
-        const unsigned key = cand ? (0x80000000u | (hi & 0x7fffffe0u) | (unsigned)(31 - r)) : 0u;
-        const unsigned kmax = (F & kFastXNoSearch) ? (key | (unsigned)(31 - (k % T))) : tile_max_key<T>(key, t);
-        int ipiv = (31 - (int)(kmax & 31u)) & (T - 1);   // (inactive tiles: in range, unused)
-        // Another candidate with the same truncated key: the lane order may not
-        // be the exact order (R1/R2).  No branch here: the tile is redone by
-        // the safe kernel (flag checked once after the last step).
-        redo = redo || (cand && ((key | 31u) == (kmax | 31u)) && r != ipiv);
-        // line 12: the pivot (and its reciprocal)
-        const bool isp = (r == ipiv) && row_ok;
-        if (isp) tag = k + 1;                                   // line 9
-        R d, yd, u1 = R(0);
-        if constexpr (HYB) {
-            // critical-path values straight from the pivot lane (warp-uniform
-            // source), issued before the row publish; the rest of the pivot
-            // row (columns >= k+2) goes through shared memory.
-            d = __shfl_sync(kFull, a[k], ipiv);
-            if constexpr (k + 1 < M) u1 = __shfl_sync(kFull, a[k + 1], ipiv);
-            if constexpr (PRE) yd = __shfl_sync(kFull, y, ipiv);
-            else yd = Num<R>::rcp_refine(d);
-            if constexpr (k + 2 < M) {
-                constexpr int j0 = (k + 2) & ~1;
+        const unsigned key = cand ? ((Num<R>::key_hi(a[k]) & 0x7fffffe0u) | lanebits) : 0u;
+        const unsigned kmax = tile_max_key<T>(key, t);
+        const int ipiv = (31 - (int)(kmax & 31u)) & (T - 1);   // (inactive tiles: in range, unused)
+        // line 12: the pivot d (and its reciprocal yd)
+        R d, yd;
+        if constexpr (W32) {
+            d = bcast(a[k], ipiv);
+            yd = PRE ? bcast(y, ipiv) : Num<R>::rcp_refine(d);
+        } else {
+            // publish the pivot row (from column k: d is read back from it)
+            R *buf = sm.row + tbase;
+            const bool isp = (r == ipiv) && row_ok;
+            if constexpr (sizeof(R) == 8 && T > 1) {
+                constexpr int j0 = k & ~1;
                 static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
                     constexpr int j = j0 + 2 * decltype(pc)::value;
                     if constexpr (j + 1 < M) st_shared_pred(isp, buf + j, a[j], a[j + 1]);
                     else st_shared_pred(isp, buf + j, a[j]);
                 });
-            }
-            __syncwarp();
-        } else if constexpr (W32) {
-            d = __shfl_sync(kFull, a[k], ipiv);
-            if constexpr (PRE) yd = __shfl_sync(kFull, y, ipiv);
-            else yd = Num<R>::rcp_refine(d);
-        } else {
-            // publish the pivot row (from column k: d is read back from it)
-            if constexpr (sizeof(R) == 8 && T > 1) {
-                constexpr int j0 = k & ~1;
-                static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
-                    constexpr int j = j0 + 2 * decltype(pc)::value;
-                    constexpr bool pub = (F & kFastXNoPub) == 0 && ((F & kFastXOnePair) == 0 || j == j0);
-                    const bool who = (F & kFastXAllLanes) ? true : isp;
-                    if constexpr (pub) {
-                        if constexpr (j + 1 < M) st_shared_pred(who, buf + j, a[j], a[j + 1]);
-                        else st_shared_pred(who, buf + j, a[j]);
-                    }
-                });
             } else if constexpr (sizeof(R) == 4 && T >= 4) {
-                // fp32: 16-B quads (4x fewer one-lane stores than scalars)
                 constexpr int j0 = k & ~3;
                 static_for<0, (M - j0 + 3) / 4>([&](auto pc) {
                     constexpr int j = j0 + 4 * decltype(pc)::value;
@@ -242,104 +374,79 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
                 });
             }
             __syncwarp();
-            if constexpr (PRE) {
-                if constexpr (sizeof(R) == 8) {
-                    const double2 p2 = *reinterpret_cast<const double2 *>(sm.slot + 2 * (tbase + ipiv));
-                    d = p2.x;
-                    yd = p2.y;
-                } else {
-                    const float2 p2 = *reinterpret_cast<const float2 *>(sm.slot + 2 * (tbase + ipiv));
-                    d = p2.x;
-                    yd = p2.y;
-                }
-            } else {
-                d = buf[k];
-                yd = (F & kFastXNoDiv) ? d : Num<R>::rcp_refine(d);
-            }
+            d = buf[k];
+            yd = Num<R>::rcp_refine(d);
         }
-        const bool sing = (Num<R>::key_hi(d) == 0u) && (Num<R>::key_lo(d) == 0u);   // R4
-        // line 13 (SCAL): rows that must not change divide 1 by 1 and use l = +0.
+        // A candidate strictly larger than the chosen pivot: the truncated
+        // key was ambiguous -> exact redo (both finite here, R2 order).
+        redo = redo || (cand && (fabs(a[k]) > fabs(d)));
+        if ((r == ipiv) && row_ok) tag = k + 1;                    // line 9
+        const bool sing = (d == R(0));                              // R4: all candidates +-0
+        // line 13 (SCAL), then lines 14-15 (GER) on the rows still unpivoted
         const bool upd = (tag == 0) && !sing;
         bool bad = false;
-        const R q = (F & kFastXNoDiv) ? a[k] * d : Num<R>::div_pre_flag(a[k], d, yd, bad);
+        const R q = Num<R>::div_nz_flag(a[k], d, yd, bad);
         redo = redo || (upd && bad);
         const R l = upd ? q : R(0);
         if (upd) a[k] = q;
         if (sing && inf == 0) inf = k + 1;
-        // lines 14-15 (GER), branch-free
-        if constexpr (HYB) {
-            if constexpr (k + 1 < M) a[k + 1] = Num<R>::fma(-l, u1, a[k + 1]);
-            if constexpr (((k + 2) & 1) && k + 2 < M) a[k + 2] = Num<R>::fma(-l, buf[k + 2], a[k + 2]);
-            constexpr int g0 = (k + 3) & ~1;
-            static_for<0, (g0 < M ? (M - g0 + 1) / 2 : 0)>([&](auto pc) {
-                constexpr int j = g0 + 2 * decltype(pc)::value;
-                if constexpr (j + 1 < M) {
-                    if constexpr (sizeof(R) == 8) {
+        if constexpr (W32) {
+            static_for<k + 1, M>([&](auto jc) {
+                constexpr int j = decltype(jc)::value;
+                if constexpr ((F & kVol) != 0) a[j] = vfma(-l, vbcast(a[j], ipiv), a[j]);
+                else a[j] = Num<R>::fma(-l, bcast(a[j], ipiv), a[j]);
+            });
+        } else {
+            const R *buf = sm.row + tbase;
+            if constexpr (sizeof(R) == 8 && T > 1) {
+                if constexpr ((k + 1) & 1) {
+                    if constexpr (k + 1 < M) a[k + 1] = Num<R>::fma(-l, buf[k + 1], a[k + 1]);
+                }
+                constexpr int j0 = (k + 2) & ~1;
+                static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
+                    constexpr int j = j0 + 2 * decltype(pc)::value;
+                    if constexpr (j + 1 < M) {
                         const double2 u = *reinterpret_cast<const double2 *>(buf + j);
                         a[j] = Num<R>::fma(-l, u.x, a[j]);
                         a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
                     } else {
-                        const float2 u = *reinterpret_cast<const float2 *>(buf + j);
+                        a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                    }
+                });
+            } else if constexpr (sizeof(R) == 4 && T >= 4) {
+                constexpr int g0 = (k + 4) & ~3;            // first quad after column k
+                static_for<k + 1, (g0 < M ? g0 : M)>([&](auto jc) {
+                    constexpr int j = decltype(jc)::value;
+                    a[j] = Num<R>::fma(-l, buf[j], a[j]);
+                });
+                static_for<0, (g0 < M ? (M - g0 + 3) / 4 : 0)>([&](auto pc) {
+                    constexpr int j = g0 + 4 * decltype(pc)::value;
+                    if constexpr (j + 3 < M) {
+                        const float4 u = *reinterpret_cast<const float4 *>(buf + j);
                         a[j] = Num<R>::fma(-l, u.x, a[j]);
                         a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
+                        a[j + 2] = Num<R>::fma(-l, u.z, a[j + 2]);
+                        a[j + 3] = Num<R>::fma(-l, u.w, a[j + 3]);
+                    } else {
+                        static_for<j, M>([&](auto jc) {
+                            constexpr int jj = decltype(jc)::value;
+                            a[jj] = Num<R>::fma(-l, buf[jj], a[jj]);
+                        });
                     }
-                } else {
+                });
+            } else {
+                static_for<k + 1, M>([&](auto jc) {
+                    constexpr int j = decltype(jc)::value;
                     a[j] = Num<R>::fma(-l, buf[j], a[j]);
-                }
-            });
-        } else if constexpr (W32) {
-            static_for<k + 1, M>([&](auto jc) {
-                constexpr int j = decltype(jc)::value;
-                const R u = __shfl_sync(kFull, a[j], ipiv);
-                a[j] = Num<R>::fma(-l, u, a[j]);
-            });
-        } else if constexpr (sizeof(R) == 8 && T > 1) {
-            if constexpr ((k + 1) & 1) {
-                if constexpr (k + 1 < M) a[k + 1] = Num<R>::fma(-l, buf[k + 1], a[k + 1]);
+                });
             }
-            constexpr int j0 = (k + 2) & ~1;
-            static_for<0, (M - j0 + 1) / 2>([&](auto pc) {
-                constexpr int j = j0 + 2 * decltype(pc)::value;
-                if constexpr (j + 1 < M) {
-                    const double2 u = *reinterpret_cast<const double2 *>(buf + j);
-                    a[j] = Num<R>::fma(-l, u.x, a[j]);
-                    a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
-                } else {
-                    a[j] = Num<R>::fma(-l, buf[j], a[j]);
-                }
-            });
-        } else if constexpr (sizeof(R) == 4 && T >= 4) {
-            constexpr int g0 = (k + 4) & ~3;            // first quad after column k
-            static_for<k + 1, (g0 < M ? g0 : M)>([&](auto jc) {
-                constexpr int j = decltype(jc)::value;
-                a[j] = Num<R>::fma(-l, buf[j], a[j]);
-            });
-            static_for<0, (g0 < M ? (M - g0 + 3) / 4 : 0)>([&](auto pc) {
-                constexpr int j = g0 + 4 * decltype(pc)::value;
-                if constexpr (j + 3 < M) {
-                    const float4 u = *reinterpret_cast<const float4 *>(buf + j);
-                    a[j] = Num<R>::fma(-l, u.x, a[j]);
-                    a[j + 1] = Num<R>::fma(-l, u.y, a[j + 1]);
-                    a[j + 2] = Num<R>::fma(-l, u.z, a[j + 2]);
-                    a[j + 3] = Num<R>::fma(-l, u.w, a[j + 3]);
-                } else {
-                    static_for<j, M>([&](auto jc) {
-                        constexpr int jj = decltype(jc)::value;
-                        a[jj] = Num<R>::fma(-l, buf[jj], a[jj]);
-                    });
-                }
-            });
-        } else {
-            static_for<k + 1, M>([&](auto jc) {
-                constexpr int j = decltype(jc)::value;
-                a[j] = Num<R>::fma(-l, buf[j], a[j]);
-            });
+            __syncwarp();
         }
-        if constexpr (!W32 && !DBL) __syncwarp();
     });
-    // Tiles that hit a pivot ambiguity or a slow-path quotient are redone by
-    // the safe kernel from the (still untouched) input.
-    if constexpr ((F & (kFastXNoPub | kFastXNoDiv | kFastXNoSearch | kFastXAllLanes | kFastXOnePair)) != 0) redo = (tag == -7);   // ablation: keep the write-back
+    // Output test of the zero-multiplier argument (header comment).
+    static_for<0, M>([&](auto jc) { redo = redo || !fast_ok(a[decltype(jc)::value]); });
+    // Tiles that hit a pivot ambiguity, a slow-path quotient or a failed
+    // output test are redone by the safe kernel from the (still untouched) input.
     if (tile_bits<T>(__ballot_sync(kFull, redo && tile_ok), tbase) != 0u) {
         if (tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
         return;
@@ -357,49 +464,52 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
 }
 
 template <typename R, int M, int MHI, int F, class AfterLoad>
-__device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const R *S, const int64_t *vec_off,
-                                                    int32_t *piv, int32_t *info, int32_t *safe_list,
-                                                    unsigned *safe_count, FastSmem<R> &sm, AfterLoad &&after_load) {
+__device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const R *S, int32_t *piv, int32_t *info,
+                                                    int32_t *safe_list, unsigned *safe_count, FastSmem<R> &sm,
+                                                    AfterLoad &&after_load) {
     if (tk.m == M) {
         constexpr int T = tile_width(M);
-        getrf_fast_tile<R, M, F>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), vec_off, piv, info,
-                                 safe_list, safe_count, sm, after_load);
+        getrf_fast_tile<R, M, F>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info, safe_list,
+                                 safe_count, sm, after_load);
     } else {
         if constexpr (M < MHI)
-            getrf_fast_dispatch<R, M + 1, MHI, F>(A, tk, S, vec_off, piv, info, safe_list, safe_count, sm,
-                                                  after_load);
+            getrf_fast_dispatch<R, M + 1, MHI, F>(A, tk, S, piv, info, safe_list, safe_count, sm, after_load);
     }
 }
 
-// Task indices in two stages so no load waits on the one before it inside
-// an iteration: getrf_fetch_idx (order[]) runs three tasks ahead,
-// getrf_fetch_off (val_off/vec_off of the block found one iteration earlier)
-// two tasks ahead.
+// Task schedule.  Tasks are enumerated bin by bin (orders MLO..MHI); warp w
+// takes tasks w, w + nwarps, ...  task_order() gives the order m of a task and
+// the index of this lane's tile's block in the plan's `order` array.
 template <int NM>
-__device__ __forceinline__ FTask getrf_fetch_idx(int64_t task, int64_t ntask, int mlo, const int64_t *s_pref,
-                                                 const int64_t *s_first, const int64_t *s_last,
-                                                 const int32_t *__restrict__ order) {
-    FTask tk;
-    tk.m = 0;
-    tk.ok = false;
-    tk.blk = 0;
-    tk.lo = 0;
-    tk.vo = 0;
-    if (task >= ntask) return tk;
+__device__ __forceinline__ int task_order(int64_t task, int mlo, const int64_t *s_pref, const int64_t *s_first,
+                                          const int64_t *s_last, int64_t &idx) {
     int i = 0;
     while (i + 1 < NM && s_pref[i + 1] <= task) ++i;
     const int m = mlo + i;
-    const int64_t idx = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m) + (threadIdx.x & 31) / tile_width(m);
-    tk.m = m;
-    tk.ok = idx < s_last[i];
-    tk.blk = tk.ok ? __ldg(order + idx) : 0;
-    return tk;
+    idx = s_first[i] + (task - s_pref[i]) * tiles_per_warp(m) + (threadIdx.x & 31) / tile_width(m);
+    if (idx >= s_last[i]) idx = -1;
+    return m;
 }
-__device__ __forceinline__ void getrf_fetch_off(FTask &tk, const int64_t *__restrict__ val_off,
-                                                const int64_t *__restrict__ vec_off) {
-    tk.lo = tk.ok ? __ldg(val_off + tk.blk) : 0;
-    tk.vo = tk.ok ? __ldg(vec_off + tk.blk) : 0;
+
+// Per-warp ring of upcoming tasks in shared memory, filled by cp.async
+// (LDGSTS: global -> shared without registers), so the index chain
+// order[] -> val_off/vec_off of tasks two and three ahead costs no registers
+// during the factorization.  Slot s, tile t: the tile's block id (-1: no
+// block), val_off and vec_off (written by the tile's lane 0).
+template <int G>                             // G = blocks (tiles) per task
+struct TaskRing {
+    int64_t lo[4][G];
+    int64_t vo[4][G];
+    int32_t blk[4][G];
+};
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 // Stage task tk's blocks into the warp's buffer S: tile t's block (m*m
 // elements, rounded up to 16 B -- the rounding stays inside the block's
@@ -417,15 +527,12 @@ __device__ __forceinline__ void getrf_stage(R *A, const FTask &tk, R *S, uint64_
     if (tk.ok && (lane % T) == 0) bulk_g2s(S + (lane / T) * stage_stride<R>(T), A + tk.lo, bytes, bar);
 }
 
-// One size class [MLO, MHI].  Tasks enumerated bin by bin; warp w takes tasks
-// w, w + nwarps, ...  Each warp owns an 8-KB staging buffer: while it factors
-// task i from registers, the bulk copy of task i+1 is in flight (and task
-// i+2's indices), so the block load no longer waits on HBM latency.
-#ifndef BJ_FAST_MINB
-#define BJ_FAST_MINB(R) (sizeof(R) == 8 ? 3 : 4)   // scripts/micro/getrf_bench.cu (B200): fp64 12 warps/SM beat 16, 20; fp32 16
-#endif
+// One size class [MLO, MHI], persistent.  Each warp owns an 8-KB staging
+// buffer: while it factors task i from registers, the bulk copy of task i+1
+// is in flight (and the indices of tasks i+2, i+3 in the ring), so the block
+// load does not wait on HBM latency.
 template <typename R, int MLO, int MHI, int F = BJ_FAST_DEFAULT>
-__global__ void __launch_bounds__(kFastThreads, BJ_FAST_MINB(R))
+__global__ void __launch_bounds__(kFastThreads, fast_min_blocks<R>(F, MHI))
 k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off,
              int32_t *__restrict__ piv, int32_t *__restrict__ info, const int32_t *__restrict__ order,
              const int64_t *__restrict__ bin_start, int32_t *__restrict__ safe_list,
@@ -433,9 +540,12 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     constexpr int NM = MHI - MLO + 1;
     __shared__ int64_t s_pref[NM + 1], s_first[NM], s_last[NM];
     __shared__ __align__(16) FastSmem<R> s_warp[kFastThreads / 32];
-    __shared__ __align__(128) R s_stage[kFastThreads / 32][32 * 32];
+    __shared__ __align__(128) R s_stage[kFastThreads / 32][stage_elems<R>(MLO, MHI)];
+    constexpr int G = tiles_per_warp(MLO);
+    __shared__ __align__(16) TaskRing<G> s_ring[kFastThreads / 32];
     __shared__ __align__(8) uint64_t s_bar[kFastThreads / 32];
     const int w = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         int64_t acc = 0;
         for (int i = 0; i < NM; ++i) {
@@ -449,62 +559,151 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
         }
         s_pref[NM] = acc;
     }
-    if ((threadIdx.x & 31) == 0) mbar_init(&s_bar[w], 1);
+    if (lane == 0) mbar_init(&s_bar[w], 1);
+    // Programmatic dependent launch: the next order's kernel may start filling
+    // SMs as this one's CTAs retire (the kernels touch disjoint blocks); each
+    // kernel waits for its predecessor before it exits, so stream order holds
+    // transitively for whatever is launched after the chain.
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     __syncthreads();
     const int64_t ntask = s_pref[NM];
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     FastSmem<R> &sm = s_warp[w];
     R *S = s_stage[w];
+    TaskRing<G> &ring = s_ring[w];
     uint64_t *bar = &s_bar[w];
     // Warp index through a warp reduction: the compiler then treats task and
     // order m as warp-uniform and emits plain SHFL/REDUX/VOTE in the
     // size-specialised code instead of collective-emulation sequences.
     const int64_t warp = __reduce_max_sync(kFull, (unsigned)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5));
-    FTask cur = getrf_fetch_idx<NM>(warp, ntask, MLO, s_pref, s_first, s_last, order);
-    FTask nxt = getrf_fetch_idx<NM>(warp + nwarps, ntask, MLO, s_pref, s_first, s_last, order);
-    FTask nn = getrf_fetch_idx<NM>(warp + 2 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
-    getrf_fetch_off(cur, val_off, vec_off);
-    getrf_fetch_off(nxt, val_off, vec_off);
-    getrf_stage(A, cur, S, bar);
+    if (warp >= ntask) {
+        asm volatile("griddepcontrol.wait;" ::: "memory");
+        return;
+    }
+    // prologue: indices of tasks 0..2 and offsets of tasks 0..1 (plain loads)
+    // a lane's tile for a task of order m is lane / tile_width(m); ring
+    // entries are written by the tile's first lane (lane % T == 0)
+    auto tile_of = [&](int64_t t) {
+        int64_t idx;
+        const int m = t < ntask ? task_order<NM>(t, MLO, s_pref, s_first, s_last, idx) : MLO;
+        return lane / tile_width(m);
+    };
+    auto writer = [&](int64_t t) {
+        int64_t idx;
+        const int m = t < ntask ? task_order<NM>(t, MLO, s_pref, s_first, s_last, idx) : MLO;
+        return (lane % tile_width(m)) == 0;
+    };
+    for (int q = 0; q < 3; ++q) {
+        const int64_t t = warp + q * nwarps;
+        int64_t idx = -1;
+        if (t < ntask) task_order<NM>(t, MLO, s_pref, s_first, s_last, idx);
+        if (writer(t)) {
+            const int g = tile_of(t);
+            const int32_t blk = idx >= 0 ? __ldg(order + idx) : -1;
+            ring.blk[q][g] = blk;
+            if (q < 2) {
+                ring.lo[q][g] = blk >= 0 ? __ldg(val_off + blk) : 0;
+                ring.vo[q][g] = blk >= 0 ? __ldg(vec_off + blk) : 0;
+            }
+        }
+    }
+    auto slot_task = [&](int64_t t, int q) {
+        FTask tk;
+        int64_t idx;
+        tk.m = t < ntask ? task_order<NM>(t, MLO, s_pref, s_first, s_last, idx) : 0;
+        const int g = tile_of(t);
+        tk.blk = ring.blk[q][g];
+        tk.ok = tk.m != 0 && tk.blk >= 0;
+        tk.lo = ring.lo[q][g];
+        tk.vo = ring.vo[q][g];
+        return tk;
+    };
+    __syncwarp();
+    getrf_stage(A, slot_task(warp, 0), S, bar);
     unsigned parity = 0;
+    int q0 = 0;
     for (int64_t task = warp; task < ntask; task += nwarps) {
-        const FTask n3 = getrf_fetch_idx<NM>(task + 3 * nwarps, ntask, MLO, s_pref, s_first, s_last, order);
-        getrf_fetch_off(nn, val_off, vec_off);
+        const int q1 = (q0 + 1) & 3, q2 = (q0 + 2) & 3, q3 = (q0 + 3) & 3;
+        // ring: offsets of task+2 (its block id landed one iteration ago), block id of task+3
+        cp_async_wait_all();
+        __syncwarp();                        // ring entries of other lanes (tile writers) visible
+        {
+            const int64_t t2 = task + 2 * nwarps, t3 = task + 3 * nwarps;
+            if (writer(t2)) {
+                const int g = tile_of(t2);
+                const int32_t b2 = ring.blk[q2][g];
+                if (b2 >= 0) {
+                    cp_async8(&ring.lo[q2][g], val_off + b2);
+                    cp_async8(&ring.vo[q2][g], vec_off + b2);
+                }
+            }
+            if (writer(t3)) {
+                const int g = tile_of(t3);
+                int64_t idx = -1;
+                if (t3 < ntask) task_order<NM>(t3, MLO, s_pref, s_first, s_last, idx);
+                if (idx >= 0) cp_async4(&ring.blk[q3][g], order + idx);
+                else ring.blk[q3][g] = -1;
+            }
+            cp_async_commit();
+        }
         mbar_wait_warp(bar, parity);
         parity ^= 1u;
+        const FTask cur = slot_task(task, q0);
         auto after_load = [&]() {
             __syncwarp();                 // every lane has its block in registers
             fence_proxy_async_smem();
-            getrf_stage(A, nxt, S, bar);
+            getrf_stage(A, slot_task(task + nwarps, q1), S, bar);
         };
-        getrf_fast_dispatch<R, MLO, MHI, F>(A, cur, S, vec_off, piv, info, safe_list, safe_count, sm, after_load);
-        cur = nxt;
-        nxt = nn;
-        nn = n3;
+        getrf_fast_dispatch<R, MLO, MHI, F>(A, cur, S, piv, info, safe_list, safe_count, sm, after_load);
+        q0 = q1;
     }
+    cp_async_wait_all();
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
+// Launch grid per (kernel, device): resident CTAs per SM x SMs.
+template <typename K>
+int persistent_grid(K kernel, int threads) {
+    static int cached[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (cached[dev] == 0) {
+        int per_sm = 0;
+        cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0);
+        cached[dev] = (per_sm < 1 ? 1 : per_sm) * sm_count();
+    }
+    return cached[dev];
+}
+
+// Launch with programmatic stream serialization (PDL, see k_getrf_fast).
 template <typename R, int MLO, int MHI>
 bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
                             const PlanView &p, int32_t *safe_list, unsigned *safe_count, cudaStream_t s) {
-    static int grid = 0;
-    if (grid == 0) {
-        int per_sm = 0;
-        cudaFuncSetAttribute(k_getrf_fast<R, MLO, MHI>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrf_fast<R, MLO, MHI>, kFastThreads, 0);
-        grid = (per_sm < 1 ? 1 : per_sm) * sm_count();
-    }
-    k_getrf_fast<R, MLO, MHI><<<grid, kFastThreads, 0, s>>>(A, val_off, vec_off, piv, info, p.order, p.bin_start,
-                                                            safe_list, safe_count);
-    BJ_LAUNCH_CHECK();
+    auto kern = k_getrf_fast<R, MLO, MHI>;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(persistent_grid(kern, kFastThreads));
+    cfg.blockDim = dim3(kFastThreads);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    BJ_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, A, val_off, vec_off, piv, info, (const int32_t *)p.order,
+                                   (const int64_t *)p.bin_start, safe_list, safe_count));
+    ::bj::count_launch();
     return BJ_OK;
 }
 
-// Safe path: blocks whose entries violate the fast path's precondition (-0,
-// non-finite, |a| >= 2^990).  The plain algorithm of Fig. 1 bottom with the
-// block in shared memory (row stride 33, lane r = row r, runtime m), explicit
-// predication of pivoted rows, exact 64-bit pivot keys: bit-identical to the
-// oracle for every input.  Rarely used, so it favours simplicity.
+// Safe path: blocks whose entries violate the fast path's precondition, or
+// whose pivot search was ambiguous in the truncated key.  The plain algorithm
+// of Fig. 1 bottom with the block in shared memory (row stride 33, lane r =
+// row r, runtime m), explicit predication of pivoted rows, exact 64-bit pivot
+// keys, IEEE division: bit-identical to the oracle for every input.  Rarely
+// used, so it favours simplicity.
 template <typename R>
 __global__ void __launch_bounds__(128)
 k_getrf_safe(R *A, const int32_t *__restrict__ sizes, const int64_t *__restrict__ val_off,

@@ -91,22 +91,69 @@ void run(Batch &b, const char *name, int64_t tot) {
            cudaGetErrorString(cudaGetLastError()));
 }
 
+
+template <int M, int F>
+void launch_one(Batch &b) {
+    auto kern = k_getrf_fast<double, M, M, F>;
+    static int grid = 0;
+    if (!grid) {
+        int per_sm = 0;
+        cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFastThreads, 0);
+        grid = per_sm * sm_count();
+        printf("   M=%d occ %d warps/SM\n", M, per_sm * 4);
+    }
+    kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt);
+}
+template <int M, int F>
+void launch_range(Batch &b) {
+    launch_one<M, F>(b);
+    if constexpr (M < 32) launch_range<M + 1, F>(b);
+}
+template <int F>
+void run_perm(Batch &b, const char *name, int64_t tot) {
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    std::vector<float> ts;
+    unsigned deferred = 0;
+    for (int rep = 0; rep < 6; ++rep) {
+        cudaMemcpy(b.A, b.A0, tot * 8, cudaMemcpyDeviceToDevice);
+        cudaMemset(b.cnt, 0, 4);
+        cudaEventRecord(e0);
+        launch_range<17, F>(b);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        if (rep) ts.push_back(ms);
+    }
+    cudaMemcpy(&deferred, b.cnt, 4, cudaMemcpyDeviceToHost);
+    std::sort(ts.begin(), ts.end());
+    printf("%-28s F=%2d per-order kernels  med %8.1f us  min %8.1f us  %7.1f GB/s  deferred=%u err=%s\n", name, F,
+           ts[ts.size() / 2] * 1e3, ts[0] * 1e3, b.bytes / (ts[ts.size() / 2] * 1e-3) / 1e9, deferred,
+           cudaGetErrorString(cudaGetLastError()));
+}
+
+template <int M>
+void per_m() {
+    Batch b = make(34500, M, M);
+    int64_t tot = 34500LL * ((M * M + 1) / 2 * 2);
+    char n[64];
+    snprintf(n, sizeof n, "M=%d 34.5k panel 2", M);
+    run<M, M, 8>(b, n, tot);
+    snprintf(n, sizeof n, "M=%d 34.5k panel 2 PRE", M);
+    run<M, M, 9>(b, n, tot);
+    snprintf(n, sizeof n, "M=%d 34.5k panel 2 PRE 16w", M);
+    run<M, M, 9 | 256>(b, n, tot);
+}
 int main() {
-    {
-        Batch b = make(40000, 32, 32);
-        int64_t tot = 40000LL * 1024;
-        run<32, 32, 0>(b, "C2 40k x 32", tot);
-        run<32, 32, 1>(b, "C2 40k x 32", tot);
-
-    }
-    {
-        const int64_t nb = 552000;
-        Batch b = make(nb, 17, 32);
-        int64_t tot = 0;
-        for (int64_t i = 0; i < nb; ++i) tot += (b.m_of[i] * b.m_of[i] + 1) / 2 * 2;
-        run<17, 32, 0>(b, "mix 17..32 552k", tot);
-        run<17, 32, 1>(b, "mix 17..32 552k", tot);
-
-    }
+    setvbuf(stdout, NULL, _IONBF, 0);
+    per_m<17>();
+    per_m<18>();
+    per_m<20>();
+    per_m<22>();
+    per_m<24>();
+    per_m<26>();
+    per_m<28>();
+    per_m<30>();
+    per_m<32>();
     return 0;
 }
