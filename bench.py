@@ -60,6 +60,14 @@ def algorithmic_bytes(sizes: np.ndarray, dt) -> tuple[int, int]:
     return getrf, getrs
 
 
+def fused_bytes(sizes: np.ndarray, dt) -> int:
+    """bj_gesv_vbatched per block: A read + L\\U written (2 s m^2), b read + x
+    written (2 s m), perm (4 m), info (4), val_off + vec_off (16)."""
+    s = esize(dt)
+    m = sizes.astype(np.int64)
+    return int((2 * s * m * m + 2 * s * m + 4 * m + 20).sum())
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -309,9 +317,7 @@ def run_ours(args, ws, rank, local):
 
     stream = torch.cuda.current_stream()
 
-    def one_step(values, evs=None):
-        vec = base.vec_off
-        val = base.val_off
+    def one_step(values, fused, evs=None):
         if evs is not None:
             evs[0].record(stream)
         v2, l2 = bj.layout(sizes, dt)                       # a1 (recomputed per step)
@@ -319,65 +325,64 @@ def run_ours(args, ws, rank, local):
         batch = bj.Batch(sizes, v2, l2, values)
         if evs is not None:
             evs[1].record(stream)
-        bj.getrf(batch, piv, info, plan=plan)               # a3
-        if evs is not None:
-            evs[2].record(stream)
-        bj.getrs(batch, piv, rhs, x, plan=plan)             # a4
-        if evs is not None:
-            evs[3].record(stream)
+        if fused:
+            bj.gesv(batch, piv, info, rhs, x, plan=plan)    # a3 + a4 fused (bj_gesv_vbatched)
+            if evs is not None:
+                evs[2].record(stream)
+                evs[3].record(stream)
+        else:
+            bj.getrf(batch, piv, info, plan=plan)           # a3
+            if evs is not None:
+                evs[2].record(stream)
+            bj.getrs(batch, piv, rhs, x, plan=plan)         # a4
+            if evs is not None:
+                evs[3].record(stream)
         return plan
 
-    # warm-up
-    keep = []
-    for i in range(args.warmup):
-        one_step(pool[i % pool_n]).close()     # stream-ordered free, no sync
-    barrier(ws)
-    for p in keep:
-        p.close()
-    keep = []
-    for i in range(min(args.warmup, pool_n)):                # restore used copies
-        pool[i].copy_(base.values)
-    barrier(ws)
-
-    # timed region(s): chunks of at most pool_n steps, restore between chunks
-    done = 0
-    t_total_ms = 0.0
-    per = []
-    bj.launch_count_reset()
-    launches = 0
-    sampler = ClockSampler(local)
-    with sampler:
-        while done < args.steps:
-            n = min(pool_n, args.steps - done)
-            evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(n)]
-            barrier(ws)
-            start = torch.cuda.Event(enable_timing=True)
-            end = torch.cuda.Event(enable_timing=True)
-            bj.launch_count_reset()
-            start.record(stream)
-            for i in range(n):
-                one_step(pool[i], evs[i]).close()
-            end.record(stream)
-            launches += bj.launch_count()
-            barrier(ws)
-            t_total_ms += start.elapsed_time(end)
-            for e in evs:
-                per.append((e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[2].elapsed_time(e[3])))
-            for p in keep:
-                p.close()
-            keep = []
-            done += n
-            if done < args.steps:
-                for i in range(min(n, pool_n)):
+    def timed(fused):
+        """W warm-up steps, then K timed steps (each on its own pristine copy);
+        returns (total ms over K steps, per-step [plan, getrf(+solve), getrs]
+        ms, launches, clock summary)."""
+        for i in range(args.warmup):
+            one_step(pool[i % pool_n], fused).close()       # stream-ordered free, no sync
+        barrier(ws)
+        for i in range(min(args.warmup, pool_n)):           # restore used copies
+            pool[i].copy_(base.values)
+        barrier(ws)
+        done, t_total_ms, per, launches = 0, 0.0, [], 0
+        sampler = ClockSampler(local)
+        with sampler:
+            while done < args.steps:
+                n = min(pool_n, args.steps - done)
+                evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(n)]
+                barrier(ws)
+                start = torch.cuda.Event(enable_timing=True)
+                end = torch.cuda.Event(enable_timing=True)
+                bj.launch_count_reset()
+                start.record(stream)
+                for i in range(n):
+                    one_step(pool[i], fused, evs[i]).close()
+                end.record(stream)
+                launches += bj.launch_count()
+                barrier(ws)
+                t_total_ms += start.elapsed_time(end)
+                for e in evs:
+                    per.append((e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[2].elapsed_time(e[3])))
+                done += n
+                for i in range(min(n, pool_n)):              # pristine copies for what follows
                     pool[i].copy_(base.values)
-    t_ms = max_over_ranks(t_total_ms, ws)
-    per = np.array(per)
-    plan_ms, getrf_ms, getrs_ms = (float(per[:, j].mean()) for j in range(3))
-    step_each = per.sum(axis=1)
+        barrier(ws)
+        return t_total_ms, np.array(per), launches, sampler.summary()
+
+    # the separate calls (getrf + getrs: the headline step), then the fused call
+    t_sep, per_sep, launches, clocks = timed(False)
+    t_fus, per_fus, launches_fus, clocks_fus = timed(True) if not args.no_fused else (None, None, 0, None)
+    t_ms = max_over_ranks(t_sep, ws)
+    plan_ms = float(per_sep[:, 0].mean())
+    getrf_ms = max_over_ranks(float(per_sep[:, 1].mean()), ws)
+    getrs_ms = max_over_ranks(float(per_sep[:, 2].mean()), ws)
+    step_each = per_sep.sum(axis=1)
     step_med, step_min = float(np.median(step_each)), float(step_each.min())
-    getrf_ms = max_over_ranks(getrf_ms, ws)
-    getrs_ms = max_over_ranks(getrs_ms, ws)
-    clocks = sampler.summary()
 
     # correctness sentinel on the timed data (cheap): no zero pivots expected
     bad = int((info[:nb] != 0).sum().item())
@@ -393,6 +398,16 @@ def run_ours(args, ws, rank, local):
     step_bytes = getrf_bytes + getrs_bytes
     ms_per_step = t_ms / args.steps
     value = nb_total / (ms_per_step * 1e-3)
+    fused = None
+    if t_fus is not None:
+        t_fus = max_over_ranks(t_fus, ws)
+        gesv_ms = max_over_ranks(float(per_fus[:, 1].mean()), ws)
+        gesv_bytes = fused_bytes(my_sizes, dt)
+        fms = t_fus / args.steps
+        fused = {"ms_per_step": fms, "value": nb_total / (fms * 1e-3), "unit": "blocks/s",
+                 "step": "layout + plan + bj_gesv_vbatched (GETRF + GETRS fused; bit-identical outputs)",
+                 "gesv_ms": gesv_ms, "gesv_bytes": gesv_bytes,
+                 "gesv_frac": gesv_bytes / (gesv_ms * 1e-3) / 1e9 / hbm, "gpu_launches": launches_fus}
 
     # ---- e2e: the C-ABI call with HOST buffers (bj_gesv_host), copies inside
     e2e = None
@@ -433,15 +448,21 @@ def run_ours(args, ws, rank, local):
             "scaling": scaling, "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32",
             "data": "synthetic (counter-based splitmix64, generated on device)",
             "config": {"workload": desc, "nblocks_total": nb_total, "nblocks_rank0": nb, "sizes": f"U{{{lo}..{hi}}}",
-                       "step": "layout + plan + getrf + getrs",
+                       "step": "layout + plan + bj_getrf_vbatched + bj_getrs_vbatched",
                        "parallelism": f"dp{ws} (contiguous cost-balanced shards, {scaling} scaling)",
                        "l2": f"inputs larger than L2: each step factors its own pristine {copy_bytes / 1e9:.2f} GB copy"},
-            "roofline": {"bound": "hbm", "kernel": f"bj_{dom}_vbatched (size-class launches)", "achieved": achieved,
+            "roofline": {"bound": "hbm", "kernel": f"bj_{dom}_vbatched (all its launches)", "achieved": achieved,
                          "peak": hbm, "unit": "GB/s", "frac": achieved / hbm, "traffic": traffic,
-                         "peak_source": peak_src, "bytes_per_launch": dom_bytes},
+                         "peak_source": peak_src, "bytes_per_launch": dom_bytes,
+                         "bytes_formula": ("per block 2 s m^2 + 4 m + 20" if dom == "getrf"
+                                           else "per block s m^2 + 2 s m + 4 m + 16")},
+            "other_call_roofline": ({"kernel": "bj_getrs_vbatched", "frac": getrs_bytes / (getrs_ms * 1e-3) / 1e9 / hbm}
+                                    if dom == "getrf" else
+                                    {"kernel": "bj_getrf_vbatched", "frac": getrf_bytes / (getrf_ms * 1e-3) / 1e9 / hbm}),
             "step_hbm": {"algorithmic_bytes": step_bytes, "achieved_gbs": step_bytes / (ms_per_step * 1e-3) / 1e9,
                          "frac": step_bytes / (ms_per_step * 1e-3) / 1e9 / hbm},
             "breakdown_ms": {"layout_plan": plan_ms, "getrf": getrf_ms, "getrs": getrs_ms},
+            "fused_gesv": fused,
             "step_ms_rank0": {"median": step_med, "min": step_min},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
             "nonzero_info_blocks": bad,
@@ -585,6 +606,7 @@ def main():
     ap.add_argument("--block", type=int, default=0, help="C4/C5 diagonal block size (default 24)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-fused", action="store_true", help="skip the extra fused bj_gesv_vbatched measurement")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
                     help="multi-GPU batched configs: shard the config's batch (strong) or replicate it per GPU (weak)")

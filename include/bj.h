@@ -161,6 +161,20 @@ bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const voi
                             const bj_plan *plan, bj_stream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * Rows a3 + a4 fused -- factor and solve in one pass (LAPACK gesv semantics):
+ * exactly bj_getrf_vbatched(blocks, pivots, info) followed by
+ * bj_getrs_vbatched(blocks, pivots, b, x) -- same outputs, bit for bit
+ * (pivots, info, L\U in blocks->values, x) -- but each block is solved while
+ * its factors are still in registers, so the factors are not read back from
+ * memory (data kept in registers; the solve of P:218-238 follows
+ * the factorization of the same block).  b and x are packed at
+ * blocks->vec_off; x may alias b exactly.  Blocks with info != 0 get the
+ * IEEE results of the division by the zero pivot (as bj_getrs_vbatched).
+ * ------------------------------------------------------------------------- */
+bj_status bj_gesv_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const void *b, void *x,
+                           const bj_plan *plan, bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
  * Hot-path row a5 -- block-Jacobi preconditioner, section II.A:
  * setup = extract + factor every diagonal block,
  * apply   y = D^{-1} x, one GETRS per block over the segments
@@ -169,8 +183,10 @@ bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const voi
  * nblocks+1 / nblocks+1 entries; factors->values must hold
  * val_off[nblocks] elements -- size it with bj_layout_from_block_ptr first),
  * extracts into factors->values, factors in place, and keeps references to
- * factors, pivots, block_ptr and a size plan in the handle.  x and y have
- * A->nrows entries of the factor dtype (local rows); y may alias x.
+ * factors, pivots, block_ptr and a size plan in the handle.  x and y cover
+ * the rows the blocks own, relative to the first block: x[i] and y[i] belong
+ * to local row block_ptr[0] + i (i < block_ptr[nb] - block_ptr[0]; with the
+ * usual block_ptr[0] = 0 they are indexed by local row).  y may alias x.
  * ------------------------------------------------------------------------- */
 bj_status bj_create(bj_handle **handle);
 bj_status bj_setup(bj_handle *handle, const bj_csr *A, const int32_t *block_ptr,
@@ -212,7 +228,10 @@ bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t 
  * End-to-end call with HOST buffers (synchronous): copies sizes_h (nblocks),
  * blocks_h (nvalues elements, packed per bj_layout) and b_h (nvec elements)
  * to the device, runs layout + plan + GETRF + GETRS, and copies x_h (nvec),
- * pivots_h (nvec, may be NULL) and info_h (nblocks, may be NULL) back.
+ * pivots_h (nvec, may be NULL)
+ * and info_h (nblocks, may be NULL) back.  nvalues / nvec smaller than the
+ * layout of sizes_h requires (sum of round_up(m^2, 16/s) / sum of m) is
+ * BJ_ERR_ARG (checked on the host before any copy).
  * Device buffers live in `ws` and grow on demand.  Host buffers should be
  * pinned (cudaHostAlloc / torch pin_memory) for full PCIe bandwidth.
  * ------------------------------------------------------------------------- */

@@ -24,7 +24,8 @@ _STATUS = {0: "BJ_OK", -1: "BJ_ERR_ARG", -2: "BJ_ERR_BLOCK_SIZE", -3: "BJ_ERR_AL
 # every symbol include/bj.h and include/bj_synth.h declare
 EXPORTS = (
     "bj_status_string", "bj_version", "bj_layout", "bj_layout_from_block_ptr", "bj_plan_create",
-    "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_create", "bj_setup",
+    "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_gesv_vbatched",
+    "bj_create", "bj_setup",
     "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
     "bj_launch_count", "bj_launch_count_reset", "bj_supervariable_blocking",
     "bj_synth_sizes", "bj_synth_blocks", "bj_synth_rhs", "bj_synth_fem_row_ptr", "bj_synth_fem_fill",
@@ -68,6 +69,7 @@ def lib() -> ctypes.CDLL:
             "bj_extract": ([P, P, P, P], I32),
             "bj_getrf_vbatched": ([P, P, P, P, P], I32),
             "bj_getrs_vbatched": ([P, P, P, P, P, P], I32),
+            "bj_gesv_vbatched": ([P, P, P, P, P, P, P], I32),
             "bj_create": ([P], I32),
             "bj_setup": ([P, P, P, P, P, P, P], I32),
             "bj_apply": ([P, P, P, P], I32),
@@ -214,6 +216,15 @@ def getrs(batch: Batch, pivots: torch.Tensor, rhs: torch.Tensor, x: torch.Tensor
     b = batch.c()
     _check(lib().bj_getrs_vbatched(ctypes.byref(b), _p(pivots), _p(rhs), _p(x), plan.handle if plan else None,
                                    _stream(stream)), "bj_getrs_vbatched")
+
+
+def gesv(batch: Batch, pivots: torch.Tensor, info: torch.Tensor, rhs: torch.Tensor, x: torch.Tensor,
+         plan: Plan | None = None, stream=None):
+    """Rows a3 + a4 fused: in-place LU with implicit pivoting and x = A^{-1} rhs
+    per block, bit-identical to getrf() then getrs() (x may be rhs)."""
+    b = batch.c()
+    _check(lib().bj_gesv_vbatched(ctypes.byref(b), _p(pivots), _p(info), _p(rhs), _p(x),
+                                  plan.handle if plan else None, _stream(stream)), "bj_gesv_vbatched")
 
 
 @dataclass

@@ -55,13 +55,45 @@ def _sources_digest():
     return h.hexdigest()
 
 
-def _compile(job):
+def _headers_digest():
+    h = hashlib.sha256()
+    for d in (CSRC, INCLUDE):
+        for f in sorted(os.listdir(d)):
+            if f.endswith((".cuh", ".h")):
+                h.update(f.encode())
+                with open(os.path.join(d, f), "rb") as fh:
+                    h.update(fh.read())
+    return h.hexdigest()
+
+
+def _job_digest(job, headers):
+    src, defs, _ = job
+    h = hashlib.sha256()
+    h.update(headers.encode())
+    h.update(" ".join(ARCH + FLAGS + defs).encode())
+    with open(os.path.join(CSRC, src), "rb") as fh:
+        h.update(fh.read())
+    return h.hexdigest()
+
+
+def _compile(job, headers=None):
+    """Compile one object unless its sources (file + every header + flags)
+    are unchanged since the last build of that object."""
     src, defs, obj = job
     out = os.path.join(BUILD, obj)
+    stamp = out + ".digest"
+    dg = _job_digest(job, headers or _headers_digest())
+    if os.path.exists(out) and os.path.exists(stamp) and open(stamp).read() == dg:
+        log = out + ".log"
+        return obj, open(log).read() if os.path.exists(log) else ""
     cmd = [NVCC, *ARCH, *FLAGS, *defs, "-c", os.path.join(CSRC, src), "-o", out]
     p = subprocess.run(cmd, capture_output=True, text=True)
     if p.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src} {defs}:\n{p.stderr[-4000:]}")
+    with open(out + ".log", "w") as fh:
+        fh.write(p.stderr)
+    with open(stamp, "w") as fh:
+        fh.write(dg)
     return obj, p.stderr
 
 
@@ -75,8 +107,9 @@ def build(force: bool = False, jobs: int | None = None, verbose: bool = False) -
     todo = _jobs()
     n = jobs or min(len(todo), os.cpu_count() or 4)
     logs = []
+    headers = _headers_digest()
     with cf.ThreadPoolExecutor(max_workers=n) as ex:
-        for obj, log in ex.map(_compile, todo):
+        for obj, log in ex.map(lambda j: _compile(j, headers), todo):
             logs.append(f"== {obj}\n{log}")
     with open(os.path.join(BUILD, "ptxas.log"), "w") as fh:
         fh.write("\n".join(logs))

@@ -66,12 +66,12 @@ struct bj_workspace {
 // stream-ordered pool; keep freed memory in the pool (no release at stream
 // syncs) so per-call allocations never reach the driver on the hot path.
 static void pool_keep_memory() {
-    static bool done = false;
-    if (done) return;
-    done = true;
+    static bool done[64] = {false};            // per device
     int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
+    done[dev] = true;
     cudaMemPool_t pool;
-    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
         uint64_t keep = UINT64_MAX;
         cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
     }
@@ -229,6 +229,34 @@ bj_status bj_getrs_vbatched(const bj_batch *lu, const int32_t *pivots, const voi
     return st;
 }
 
+bj_status bj_gesv_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const void *b, void *x,
+                           const bj_plan *plan, bj_stream_t stream) {
+    pool_keep_memory();
+    bj_status st = check_batch(blocks, true);
+    if (st != BJ_OK) return st;
+    if (blocks->nblocks > 0 && (!pivots || !info || !b || !x)) return BJ_ERR_ARG;
+    if (plan && plan->nblocks != blocks->nblocks) return BJ_ERR_ARG;
+    if (blocks->nblocks == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    bj_plan tmp;
+    const bj_plan *p = plan;
+    if (!p) {
+        if ((st = plan_alloc_build(&tmp, blocks->nblocks, blocks->sizes, s)) != BJ_OK) {
+            plan_free_async(&tmp, s);
+            return st;
+        }
+        p = &tmp;
+    }
+    if (blocks->dtype == BJ_F64)
+        st = gesv_run<double>((double *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                              blocks->sizes, (const double *)b, (double *)x, s);
+    else
+        st = gesv_run<float>((float *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                             blocks->sizes, (const float *)b, (float *)x, s);
+    if (!plan) plan_free_async(&tmp, s);
+    return st;
+}
+
 bj_status bj_create(bj_handle **handle) {
     if (!handle) return BJ_ERR_ARG;
     bj_handle *h = new (std::nothrow) bj_handle();
@@ -321,6 +349,16 @@ bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int
     if (!ws || nb < 0 || nvalues < 0 || nvec < 0 || es == 0) return BJ_ERR_ARG;
     if (nb > 0 && (!sizes_h || !blocks_h || !b_h || !x_h)) return BJ_ERR_ARG;
     if (nb == 0) return BJ_OK;
+    {   // the caller's buffers must hold the layout of sizes_h (host arithmetic, no copy yet)
+        const int64_t q = 16 / es;
+        int64_t need_val = 0, need_vec = 0;
+        for (int64_t i = 0; i < nb; ++i) {
+            const int64_t m = sizes_h[i] > 0 ? sizes_h[i] : 0;
+            need_val += (m * m + q - 1) / q * q;
+            need_vec += m;
+        }
+        if (nvalues < need_val || nvec < need_vec) return BJ_ERR_ARG;
+    }
     cudaStream_t s = (cudaStream_t)stream;
     const size_t o_sizes = 0;
     const size_t o_vec = o_sizes + up256(sizeof(int32_t) * nb);
@@ -355,6 +393,9 @@ bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int
     p.bin_start = (int64_t *)(d + o_bins);
     if ((st = build_plan(nb, sizes, p.order, p.bin_start, s)) != BJ_OK) return st;
     bj_batch batch{nb, sizes, vec, val, d + o_A, dtype};
+    // separate calls: measured faster than the fused bj_gesv_vbatched on B200
+    // (profiles/r02: the in-register solve costs more issue slots than
+    // re-reading the factors)
     if ((st = bj_getrf_vbatched(&batch, piv, info, &p, stream)) != BJ_OK) return st;
     if ((st = bj_getrs_vbatched(&batch, piv, d + o_b, d + o_x, &p, stream)) != BJ_OK) return st;
     BJ_CUDA_TRY(cudaMemcpyAsync(x_h, d + o_x, (size_t)es * nvec, cudaMemcpyDeviceToHost, s));

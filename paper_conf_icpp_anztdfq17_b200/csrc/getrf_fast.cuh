@@ -99,6 +99,7 @@ constexpr int kMaxPanel = 4;
 template <typename R>
 struct FastSmem {
     R row[32];                                    // pivot-row buffer, T elements per tile (sub-warp tiles)
+    int pinv[32];                                 // fused solve: lane of the row at position k, per tile
     R panel[kMaxPanel][panel_stride<R>()];        // full-warp tiles: the panel's pivot rows (stale trailing part)
 };
 
@@ -125,7 +126,7 @@ __host__ __device__ constexpr int panel_width(int F) {
 template <typename R>
 __host__ __device__ constexpr int fast_min_blocks(int F, int MHI) {
     return (F & kMin3) ? 3 : (F & kMin4) ? 4 : (F & kMin6) ? 6 : (F & kMin5) ? 5
-         : (MHI * (int)sizeof(R) / 4 <= 44) ? 6 : (MHI * (int)sizeof(R) / 4 <= 52) ? 5 : 4;
+         : (sizeof(R) == 8 || MHI > 26) ? 4 : 5;
 }
 // Staging buffer per warp: one task = 32/T blocks of order <= MHI.
 template <typename R>
@@ -290,14 +291,48 @@ __device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, int &inf, b
     });
 }
 
+// Fused GETRS (bj_gesv_vbatched): the factors are still in registers -- lane
+// r holds row r of the block, which is row pos = tag-1 of L\U -- so the solve
+// of P:218-238 (b := P b, eager unit-lower solve, eager upper solve with
+// division by U(k,k); Fig. 2 bottom, R8) needs no reload of the factors.
+// Lane r starts with y_pos = b_r (b := P b), the position-k value is
+// broadcast from the lane holding position k (inverse permutation in shared
+// memory), and each lane updates only its own position, in the oracle's
+// order; rows that must not change keep their value by selection (y may hold
+// -0).  x may alias b exactly: every b is read before any x is written.
+template <typename R, int M>
+__device__ __forceinline__ void getrf_tile_solve(const R (&a)[M], int pos, bool row_ok, int r, int tbase,
+                                                 const R *b, R *x, FastSmem<R> &sm) {
+    R y = row_ok ? b[r] : R(0);
+    __syncwarp();
+    if (row_ok) sm.pinv[tbase + pos] = r;
+    __syncwarp();
+    static_for<0, M - 1>([&](auto kc) {                 // forward, unit lower
+        constexpr int k = decltype(kc)::value;
+        const R yk = __shfl_sync(kFull, y, tbase + sm.pinv[tbase + k]);
+        const R t = Num<R>::fma(a[k], -yk, y);
+        if (pos > k) y = t;
+    });
+    static_for<0, M>([&](auto kc) {                     // backward, upper
+        constexpr int k = M - 1 - decltype(kc)::value;
+        if (pos == k) y = Num<R>::div_pre(y, a[k], Num<R>::rcp_refine(a[k]));
+        if constexpr (k > 0) {
+            const R yk = __shfl_sync(kFull, y, tbase + sm.pinv[tbase + k]);
+            const R t = Num<R>::fma(a[k], -yk, y);
+            if (pos < k) y = t;
+        }
+    });
+    if (row_ok) x[pos] = y;
+}
+
 // S: this tile's block staged in shared memory by the bulk copy (column-major,
 // leading dimension M); `after_load` runs once the block is in registers
 // (it re-arms the warp's staging buffer with the next task).
-template <typename R, int M, int F, class AfterLoad>
+template <typename R, int M, int F, bool SOLVE, class AfterLoad>
 __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &tk, const R *S,
                                                 int32_t *__restrict__ piv, int32_t *__restrict__ info,
                                                 int32_t *__restrict__ safe_list, unsigned *__restrict__ safe_count,
-                                                FastSmem<R> &sm, AfterLoad &&after_load) {
+                                                const R *b, R *x, FastSmem<R> &sm, AfterLoad &&after_load) {
     constexpr int T = tile_width(M);
     constexpr bool W32 = (T == 32);
     constexpr bool PRE = W32 && (F & kPre) != 0;
@@ -446,34 +481,38 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     // Output test of the zero-multiplier argument (header comment).
     static_for<0, M>([&](auto jc) { redo = redo || !fast_ok(a[decltype(jc)::value]); });
     // Tiles that hit a pivot ambiguity, a slow-path quotient or a failed
-    // output test are redone by the safe kernel from the (still untouched) input.
-    if (tile_bits<T>(__ballot_sync(kFull, redo && tile_ok), tbase) != 0u) {
-        if (tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
-        return;
-    }
+    // output test are redone by the safe kernel from the (still untouched)
+    // input; the other tiles of the warp go on (the solve's shuffles need
+    // every lane, so no lane returns early).
+    const bool again = tile_bits<T>(__ballot_sync(kFull, redo && tile_ok), tbase) != 0u;
+    if (again && tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
+    const bool keep = tile_ok && !again;
+    const bool row_keep = keep && (r < M);
     // lines 18-19: combined row swap while off-loading L\U.
-    if (row_ok) {
-        const int pos = tag - 1;
+    const int pos = tag - 1;
+    if (row_keep) {
         static_for<0, M>([&](auto jc) {
             constexpr int j = decltype(jc)::value;
             Ab[pos + j * M] = a[j];
         });
         piv[tk.vo + pos] = r;
     }
-    if (tile_ok && r == 0) info[blk] = inf;
+    if (keep && r == 0) info[blk] = inf;
+    if constexpr (SOLVE) getrf_tile_solve<R, M>(a, pos, row_keep, r, tbase, b + tk.vo, x + tk.vo, sm);
 }
 
-template <typename R, int M, int MHI, int F, class AfterLoad>
+template <typename R, int M, int MHI, int F, bool SOLVE, class AfterLoad>
 __device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const R *S, int32_t *piv, int32_t *info,
-                                                    int32_t *safe_list, unsigned *safe_count, FastSmem<R> &sm,
-                                                    AfterLoad &&after_load) {
+                                                    int32_t *safe_list, unsigned *safe_count, const R *b, R *x,
+                                                    FastSmem<R> &sm, AfterLoad &&after_load) {
     if (tk.m == M) {
         constexpr int T = tile_width(M);
-        getrf_fast_tile<R, M, F>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info, safe_list,
-                                 safe_count, sm, after_load);
+        getrf_fast_tile<R, M, F, SOLVE>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info,
+                                        safe_list, safe_count, b, x, sm, after_load);
     } else {
         if constexpr (M < MHI)
-            getrf_fast_dispatch<R, M + 1, MHI, F>(A, tk, S, piv, info, safe_list, safe_count, sm, after_load);
+            getrf_fast_dispatch<R, M + 1, MHI, F, SOLVE>(A, tk, S, piv, info, safe_list, safe_count, b, x, sm,
+                                                         after_load);
     }
 }
 
@@ -531,12 +570,12 @@ __device__ __forceinline__ void getrf_stage(R *A, const FTask &tk, R *S, uint64_
 // buffer: while it factors task i from registers, the bulk copy of task i+1
 // is in flight (and the indices of tasks i+2, i+3 in the ring), so the block
 // load does not wait on HBM latency.
-template <typename R, int MLO, int MHI, int F = BJ_FAST_DEFAULT>
+template <typename R, int MLO, int MHI, int F = BJ_FAST_DEFAULT, bool SOLVE = false>
 __global__ void __launch_bounds__(kFastThreads, fast_min_blocks<R>(F, MHI))
 k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off,
              int32_t *__restrict__ piv, int32_t *__restrict__ info, const int32_t *__restrict__ order,
              const int64_t *__restrict__ bin_start, int32_t *__restrict__ safe_list,
-             unsigned *__restrict__ safe_count) {
+             unsigned *__restrict__ safe_count, const R *b = nullptr, R *x = nullptr) {
     constexpr int NM = MHI - MLO + 1;
     __shared__ int64_t s_pref[NM + 1], s_first[NM], s_last[NM];
     __shared__ __align__(16) FastSmem<R> s_warp[kFastThreads / 32];
@@ -654,7 +693,8 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
             fence_proxy_async_smem();
             getrf_stage(A, slot_task(task + nwarps, q1), S, bar);
         };
-        getrf_fast_dispatch<R, MLO, MHI, F>(A, cur, S, piv, info, safe_list, safe_count, sm, after_load);
+        getrf_fast_dispatch<R, MLO, MHI, F, SOLVE>(A, cur, S, piv, info, safe_list, safe_count, b, x, sm,
+                                                   after_load);
         q0 = q1;
     }
     cp_async_wait_all();
@@ -678,10 +718,11 @@ int persistent_grid(K kernel, int threads) {
 }
 
 // Launch with programmatic stream serialization (PDL, see k_getrf_fast).
-template <typename R, int MLO, int MHI>
+template <typename R, int MLO, int MHI, bool SOLVE>
 bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
-                            const PlanView &p, int32_t *safe_list, unsigned *safe_count, cudaStream_t s) {
-    auto kern = k_getrf_fast<R, MLO, MHI>;
+                            const PlanView &p, int32_t *safe_list, unsigned *safe_count, const R *b, R *x,
+                            cudaStream_t s) {
+    auto kern = k_getrf_fast<R, MLO, MHI, BJ_FAST_DEFAULT, SOLVE>;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(persistent_grid(kern, kFastThreads));
     cfg.blockDim = dim3(kFastThreads);
@@ -693,7 +734,7 @@ bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     BJ_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, A, val_off, vec_off, piv, info, (const int32_t *)p.order,
-                                   (const int64_t *)p.bin_start, safe_list, safe_count));
+                                   (const int64_t *)p.bin_start, safe_list, safe_count, b, x));
     ::bj::count_launch();
     return BJ_OK;
 }
@@ -708,7 +749,8 @@ template <typename R>
 __global__ void __launch_bounds__(128)
 k_getrf_safe(R *A, const int32_t *__restrict__ sizes, const int64_t *__restrict__ val_off,
              const int64_t *__restrict__ vec_off, int32_t *__restrict__ piv, int32_t *__restrict__ info,
-             const int32_t *__restrict__ list, const unsigned *__restrict__ count) {
+             const int32_t *__restrict__ list, const unsigned *__restrict__ count, const R *b = nullptr,
+             R *x = nullptr) {
     __shared__ R S[4][32 * 33];
     const int r = threadIdx.x & 31, w = threadIdx.x >> 5;
     R *s = S[w];
@@ -757,6 +799,22 @@ k_getrf_safe(R *A, const int32_t *__restrict__ sizes, const int64_t *__restrict_
             piv[vec_off[blk] + pos] = r;
         }
         if (r == 0) info[blk] = inf;
+        __syncwarp();
+        if (b != nullptr && r == 0) {
+            // fused solve (bj_gesv_vbatched): plain scalar GETRS from the factors
+            // just written (R8), same operations as the oracle's
+            const int64_t vo = vec_off[blk];
+            const int32_t *p = piv + vo;
+            R v[kMaxM];
+            for (int i = 0; i < m; ++i) v[i] = b[vo + p[i]];
+            for (int k = 0; k + 1 < m; ++k)
+                for (int i = k + 1; i < m; ++i) v[i] = Num<R>::fma(-Ab[i + k * m], v[k], v[i]);
+            for (int k = m - 1; k >= 0; --k) {
+                v[k] = Num<R>::div(v[k], Ab[k + k * m]);
+                for (int i = 0; i < k; ++i) v[i] = Num<R>::fma(-Ab[i + k * m], v[k], v[i]);
+            }
+            for (int i = 0; i < m; ++i) x[vo + i] = v[i];
+        }
         __syncwarp();
     }
 }

@@ -24,6 +24,9 @@ template <typename R>
 bj_status getrf_run(R *values, const int64_t *val_off, const int64_t *vec_off, int32_t *piv,
                     int32_t *info, const PlanView &plan, const int32_t *sizes, cudaStream_t s);
 template <typename R>
+bj_status gesv_run(R *values, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
+                   const PlanView &plan, const int32_t *sizes, const R *b, R *x, cudaStream_t s);
+template <typename R>
 bj_status getrs_run(const R *lu, const int64_t *val_off, const int64_t *vec_off, const int32_t *piv,
                     const R *b, R *x, const PlanView &plan, cudaStream_t s);
 

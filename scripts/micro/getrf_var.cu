@@ -21,10 +21,16 @@ __global__ void fill(double *a, int64_t n, unsigned long long seed) {
     }
 }
 
+__global__ void to_float(const double *a, float *f, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        f[i] = (float)a[i];
+}
+
 struct Batch {
     int64_t nb;
     std::vector<int> m_of;
     double *A, *A0;
+    float *Af, *Af0;
     int64_t *dvo, *dve, *dbs;
     int32_t *dord, *piv, *info, *safe;
     unsigned *cnt;
@@ -42,7 +48,7 @@ static Batch make(int64_t nb, int lo, int hi) {
     b.bytes = 0;
     for (int64_t i = 0; i < nb; ++i) {
         int m = b.m_of[i];
-        vo[i + 1] = vo[i] + (m * m + 1) / 2 * 2; ve[i + 1] = ve[i] + m; ord[i] = (int32_t)i; cntb[m]++;
+        vo[i + 1] = vo[i] + (m * m + 3) / 4 * 4; ve[i + 1] = ve[i] + m; ord[i] = (int32_t)i; cntb[m]++;
         b.bytes += 2.0 * 8 * m * m + 4 * m + 20;
     }
     int64_t acc = 0;
@@ -61,6 +67,8 @@ static Batch make(int64_t nb, int lo, int hi) {
     static int64_t tot;
     tot = vo[nb];
     cudaMemcpy(b.A, b.A0, tot * 8, cudaMemcpyDeviceToDevice);
+    cudaMalloc(&b.Af, tot * 4); cudaMalloc(&b.Af0, tot * 4);
+    to_float<<<1024, 256>>>(b.A0, b.Af0, tot);
     return b;
 }
 
@@ -132,27 +140,46 @@ void run_perm(Batch &b, const char *name, int64_t tot) {
            cudaGetErrorString(cudaGetLastError()));
 }
 
+template <int M, int F>
+void run_f(Batch &b, const char *name, int64_t tot) {
+    auto kern = k_getrf_fast<float, M, M, F>;
+    int per_sm = 0;
+    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFastThreads, 0);
+    const int grid = per_sm * sm_count();
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    std::vector<float> ts;
+    for (int rep = 0; rep < 6; ++rep) {
+        cudaMemcpy(b.Af, b.Af0, tot * 4, cudaMemcpyDeviceToDevice);
+        cudaMemset(b.cnt, 0, 4);
+        cudaEventRecord(e0);
+        kern<<<grid, kFastThreads>>>(b.Af, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        if (rep) ts.push_back(ms);
+    }
+    std::sort(ts.begin(), ts.end());
+    printf("%-28s F=%3d occ=%2d warps/SM  med %8.1f us  min %8.1f us  err=%s\n", name, F, per_sm * 4,
+           ts[ts.size() / 2] * 1e3, ts[0] * 1e3, cudaGetErrorString(cudaGetLastError()));
+}
 template <int M>
 void per_m() {
     Batch b = make(34500, M, M);
-    int64_t tot = 34500LL * ((M * M + 1) / 2 * 2);
+    int64_t tot = 34500LL * ((M * M + 3) / 4 * 4);
     char n[64];
-    snprintf(n, sizeof n, "M=%d 34.5k panel 2", M);
-    run<M, M, 8>(b, n, tot);
-    snprintf(n, sizeof n, "M=%d 34.5k panel 2 PRE", M);
-    run<M, M, 9>(b, n, tot);
-    snprintf(n, sizeof n, "M=%d 34.5k panel 2 PRE 16w", M);
-    run<M, M, 9 | 256>(b, n, tot);
+    snprintf(n, sizeof n, "fp32 M=%d 34.5k", M);
+    run_f<M, 8 | 256>(b, n, tot);
+    run_f<M, 8 | 64>(b, n, tot);
+    run_f<M, 8 | 128>(b, n, tot);
+    run_f<M, 16 | 64>(b, n, tot);
+    run_f<M, 32 | 64>(b, n, tot);
 }
 int main() {
     setvbuf(stdout, NULL, _IONBF, 0);
     per_m<17>();
-    per_m<18>();
-    per_m<20>();
     per_m<22>();
-    per_m<24>();
     per_m<26>();
-    per_m<28>();
     per_m<30>();
     per_m<32>();
     return 0;

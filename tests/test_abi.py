@@ -87,3 +87,23 @@ def test_errors_without_gpu_are_arguments(lib):
     nb = ctypes.c_int64(0)
     assert lib.bj_supervariable_blocking(ctypes.cast(csr, ctypes.c_void_p), 33, ctypes.c_void_p(16), ctypes.byref(nb),
                                          None) == -1
+
+
+def test_gesv_host_rejects_short_buffers():
+    """bj_gesv_host checks nvalues / nvec against the layout of sizes_h on the
+    host, before any device work (so this runs without a GPU)."""
+    from paper_conf_icpp_anztdfq17_b200 import bj
+    L = bj.lib()
+    ws = ctypes.c_void_p()
+    assert L.bj_workspace_create(ctypes.byref(ws)) == 0
+    sizes = np.array([3, 32, 1, 0, 7], dtype=np.int32)
+    vec, val = oracle.layout(sizes, 8)
+    need_val, need_vec = int(val[-1]), int(vec[-1])
+    A = np.zeros(need_val, np.float64)
+    b = np.zeros(need_vec, np.float64)
+    x = np.zeros(need_vec, np.float64)
+    P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+    for nvalues, nvec in ((need_val - 1, need_vec), (need_val, need_vec - 1), (0, 0)):
+        st = L.bj_gesv_host(ws, len(sizes), P(sizes), nvalues, P(A), nvec, P(b), P(x), None, None, 1, None)
+        assert st == -1, (nvalues, nvec, st)
+    L.bj_workspace_destroy(ws)

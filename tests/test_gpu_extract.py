@@ -190,3 +190,33 @@ def test_block_jacobi_handle_setup_apply(dtype):
     h.apply(y2, y2)
     torch.cuda.synchronize()
     assert torch.equal(y2, y)
+
+
+def test_block_jacobi_block_ptr_offset():
+    """bj_setup / bj_apply with block_ptr[0] != 0 (a slice of a global block
+    list): x and y are indexed relative to block_ptr[0] (include/bj.h)."""
+    nx, ny, nz = 10, 9, 8
+    g = S.FemGrid(nx, ny, nz)
+    n = g.n
+    A = bj.synth_fem(nx, ny, nz, 0, n)
+    off, b = 30, 12
+    bp = np.arange(off, n + 1, b, dtype=np.int32)
+    bp = np.unique(np.append(bp, n)).astype(np.int32)
+    bpt = torch.from_numpy(bp).cuda()
+    sizes, vec, val = bj.layout_from_block_ptr(bpt, torch.float64)
+    fac = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=torch.float64, device="cuda"))
+    rows = n - off
+    piv = torch.empty(rows, dtype=torch.int32, device="cuda")
+    info = torch.empty(len(bp) - 1, dtype=torch.int32, device="cuda")
+    h = bj.Handle()
+    h.setup(A, bpt, fac, piv, info)
+    x = torch.from_numpy(np.random.default_rng(45).uniform(-1, 1, rows)).cuda()
+    y = torch.empty_like(x)
+    h.apply(x, y)
+    torch.cuda.synchronize()
+    rp, ci, va = g.csr()
+    D, sz, vo, vl = oracle.extract(rp, ci, va, bp)
+    LU, po, io = oracle.getrf_batch(sz, vl, vo, D)
+    yo = oracle.getrs_batch(sz, vl, vo, LU, po, x.cpu().numpy())
+    assert np.array_equal(info.cpu().numpy(), io) and np.array_equal(piv.cpu().numpy(), po)
+    assert np.array_equal(bits(y.cpu().numpy()), bits(yo))

@@ -303,3 +303,74 @@ def test_c3_logical_sharding(G):
         assert torch.equal(sx.view(torch.int64), x[ve[s]: ve[e]].view(torch.int64))
         del sb, sp, si, sx
     torch.cuda.synchronize()
+
+
+def _gesv(sizes_np, dtype, kind="uniform", alias=False):
+    """bj_gesv_vbatched (fused factor + solve) against the oracle's GETRF then
+    GETRS, and against the library's own separate calls, bit for bit."""
+    npdt = NP[dtype]
+    vec, val = host_layout(sizes_np, dtype)
+    A = S.block_values(sizes_np, val, dtype=npdt, kind=kind)
+    b = S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt)
+    batch = device_batch(sizes_np, dtype, values_np=A)
+    nvec = int(vec[-1])
+    piv = torch.full((max(nvec, 1),), -7, dtype=torch.int32, device="cuda")
+    info = torch.full((max(len(sizes_np), 1),), -9, dtype=torch.int32, device="cuda")
+    bt = torch.from_numpy(b).to("cuda") if nvec else torch.zeros(1, dtype=dtype, device="cuda")
+    x = bt if alias else torch.full_like(bt, float("nan"))
+    bj.gesv(batch, piv, info, bt, x)
+    torch.cuda.synchronize()
+    LU_o, piv_o, info_o = compare_getrf(sizes_np, val, vec, A, batch.values.cpu().numpy(), piv.cpu().numpy()[:nvec],
+                                        info.cpu().numpy()[: len(sizes_np)], dtype)
+    x_o = oracle.getrs_batch(sizes_np, val, vec, LU_o, piv_o, b)
+    xd = x.cpu().numpy()[:nvec]
+    m = np.maximum(sizes_np.astype(np.int64), 0)
+    valid = np.repeat((sizes_np >= 1) & (sizes_np <= 32), m)          # entries of factored blocks
+    assert np.array_equal(np.isnan(xd[valid]), np.isnan(x_o[valid]))
+    ok = valid & np.isfinite(x_o)
+    assert np.array_equal(bits(xd[ok]), bits(x_o[ok]))
+    return A, b, vec, val, xd
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("kind", ["uniform", "int"])
+def test_gesv_every_order(dtype, kind):
+    """Fused factor + solve on every order 1..32 with ragged tails (and exact
+    ties / singular steps for integer blocks)."""
+    sizes = np.concatenate([np.full(37, m, np.int32) for m in range(1, 33)] + [np.array([0, 5, 33, 17], np.int32)])
+    _gesv(sizes, dtype, kind)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_gesv_c1_and_alias(dtype):
+    sizes = S.block_sizes(1000, 4, 16)
+    A, b, vec, val, xd = _gesv(sizes, dtype, alias=True)
+    assert backward_error(sizes, val, vec, A, b, xd) <= TOL[dtype]
+
+
+def test_gesv_c3_full_size_all_blocks():
+    """Config C3 (1M blocks) through the fused call: every block equals the
+    oracle (and hence the separate getrf + getrs calls)."""
+    nb = 1_000_000
+    dtype = torch.float64
+    sizes_d = bj.synth_sizes(nb, 4, 32)
+    batch = bj.new_batch(sizes_d, dtype)
+    bj.synth_blocks(batch)
+    b = bj.synth_rhs(batch)
+    nvec = int(batch.vec_off[-1].item())
+    piv = torch.empty(nvec, dtype=torch.int32, device="cuda")
+    info = torch.empty(nb, dtype=torch.int32, device="cuda")
+    x = torch.empty_like(b)
+    plan = bj.Plan(batch.sizes)
+    bj.gesv(batch, piv, info, b, x, plan=plan)
+    torch.cuda.synchronize()
+    sizes = S.block_sizes(nb, 4, 32)
+    vec, val = host_layout(sizes, dtype)
+    A = S.block_values_fast(sizes, val)
+    bh = S.rhs_values_fast(sizes)
+    LU_o, piv_o, info_o = oracle.getrf_batch(sizes, val, vec, A)
+    x_o = oracle.getrs_batch(sizes, val, vec, LU_o, piv_o, bh)
+    assert np.array_equal(info.cpu().numpy(), info_o)
+    assert np.array_equal(piv.cpu().numpy(), piv_o)
+    assert np.array_equal(bits(batch.values.cpu().numpy()[: len(LU_o)]), bits(LU_o))
+    assert np.array_equal(bits(x.cpu().numpy()), bits(x_o))
