@@ -69,6 +69,15 @@ def _declare(L):
         getattr(L, f"bjo_getrf_batch_{s}").restype = None
         getattr(L, f"bjo_getrs_batch_{s}").argtypes = [_i64, _p, _p, _p, _p, _p, _p, _p, _i32]
         getattr(L, f"bjo_getrs_batch_{s}").restype = None
+    for s in ("d", "s"):
+        getattr(L, f"bjo_getri_{s}").argtypes = [_i32, _p, _p]
+        getattr(L, f"bjo_getri_{s}").restype = _i32
+        getattr(L, f"bjo_gemv_{s}").argtypes = [_i32, _p, _p, _p]
+        getattr(L, f"bjo_gemv_{s}").restype = None
+        getattr(L, f"bjo_getri_batch_{s}").argtypes = [_i64, _p, _p, _p, _p, _p, _p, _i32]
+        getattr(L, f"bjo_getri_batch_{s}").restype = None
+        getattr(L, f"bjo_gemv_batch_{s}").argtypes = [_i64, _p, _p, _p, _p, _p, _p, _i32]
+        getattr(L, f"bjo_gemv_batch_{s}").restype = None
     L.bjo_layout.argtypes = [_i64, _p, _i32, _p, _p]
     L.bjo_layout.restype = None
     L.bjo_extract.argtypes = [_i64, _p, _p, _p, _i32, _i64, _i64, _p, _p, _p]
@@ -172,6 +181,60 @@ def getrs_batch(sizes, val_off, vec_off, LU, perm, b, nthreads: int = 0):
     getattr(lib(), f"bjo_getrs_batch_{s}")(nb, _ptr(sizes), _ptr(val_off), _ptr(vec_off),
                                            _ptr(LU), _ptr(perm), _ptr(b), _ptr(x), int(nthreads))
     return x[: int(vec_off[nb])]
+
+
+def getri(A: np.ndarray):
+    """Inverse of one block by Gauss-Jordan elimination with implicit partial
+    pivoting (inversion-based variant; readings R23-R26).
+    Returns (Dinv as a 2-D array Dinv[a, b], perm, info)."""
+    A = np.asarray(A)
+    m = A.shape[0]
+    s = _sfx(A.dtype)
+    buf = np.array(A, dtype=A.dtype, order="F", copy=True)
+    perm = np.zeros(max(m, 1), dtype=np.int32)
+    info = getattr(lib(), f"bjo_getri_{s}")(m, _ptr(buf), _ptr(perm))
+    return buf, perm[:m].copy(), int(info)
+
+
+def gemv(Dinv: np.ndarray, x: np.ndarray):
+    """y = Dinv x, fma chain over columns in order from +0 (R26)."""
+    Dinv = np.asarray(Dinv)
+    m = Dinv.shape[0]
+    s = _sfx(Dinv.dtype)
+    d = np.array(Dinv, order="F", copy=True)
+    xx = np.ascontiguousarray(x, dtype=Dinv.dtype)
+    y = np.zeros(max(m, 1), dtype=Dinv.dtype)
+    getattr(lib(), f"bjo_gemv_{s}")(m, _ptr(d), _ptr(xx), _ptr(y))
+    return y[:m].copy()
+
+
+def getri_batch(sizes, val_off, vec_off, values, nthreads: int = 0):
+    """Batched GJE inverse on a packed copy; returns (Dinv, perm, info)."""
+    sizes = np.ascontiguousarray(sizes, dtype=np.int32)
+    val_off = np.ascontiguousarray(val_off, dtype=np.int64)
+    vec_off = np.ascontiguousarray(vec_off, dtype=np.int64)
+    A = np.array(values, copy=True)
+    s = _sfx(A.dtype)
+    nb = sizes.shape[0]
+    perm = np.zeros(max(int(vec_off[nb]), 1), dtype=np.int32)
+    info = np.zeros(max(nb, 1), dtype=np.int32)
+    getattr(lib(), f"bjo_getri_batch_{s}")(nb, _ptr(sizes), _ptr(val_off), _ptr(vec_off),
+                                           _ptr(A), _ptr(perm), _ptr(info), int(nthreads))
+    return A, perm[: int(vec_off[nb])], info[:nb]
+
+
+def gemv_batch(sizes, val_off, vec_off, Dinv, x, nthreads: int = 0):
+    sizes = np.ascontiguousarray(sizes, dtype=np.int32)
+    val_off = np.ascontiguousarray(val_off, dtype=np.int64)
+    vec_off = np.ascontiguousarray(vec_off, dtype=np.int64)
+    Dinv = np.ascontiguousarray(Dinv)
+    s = _sfx(Dinv.dtype)
+    x = np.ascontiguousarray(x, dtype=Dinv.dtype)
+    nb = sizes.shape[0]
+    y = np.zeros(max(int(vec_off[nb]), 1), dtype=Dinv.dtype)
+    getattr(lib(), f"bjo_gemv_batch_{s}")(nb, _ptr(sizes), _ptr(val_off), _ptr(vec_off),
+                                          _ptr(Dinv), _ptr(x), _ptr(y), int(nthreads))
+    return y[: int(vec_off[nb])]
 
 
 def extract(row_ptr, col_idx, values, block_ptr, col_offset: int = 0):
