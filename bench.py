@@ -504,43 +504,64 @@ def run_fem(args, ws, rank, local):
     x = torch.rand(n, dtype=dt, device="cuda") * 2 - 1
     y = torch.empty_like(x)
     h = bj.Handle() if args.config == "C5" else None
+    hinv = bj.Handle() if args.config == "C5" else None
     napply = 100
 
     sv_bytes = 8 * (n + 1) + 4 * A.col_idx.numel() + 4 * (n // b + 2)   # row_ptr + col_idx read, block_ptr written
     sv_nb = [0]
 
-    def step(evs=None):
+    def step(evs=None, inverse=False):
         if args.config == "SV":
             sv_nb[0] = bj.supervariable_blocking(A, b).numel() - 1
         elif args.config == "C4":
             bj.extract(A, bp, out)
         else:
+            hh = hinv if inverse else h
             if evs is not None:
                 evs[0].record(stream)
-            h.setup(A, bp, out, piv, info)
+            if inverse:
+                hh.setup_inverse(A, bp, out, piv, info)      # NEXT(3): extract + GJE inverses
+            else:
+                hh.setup(A, bp, out, piv, info)              # extract + GETRF
             if evs is not None:
                 evs[1].record(stream)
             for _ in range(napply):
-                h.apply(x, y)
+                hh.apply(x, y)                               # GETRS / GEMV
 
-    for _ in range(args.warmup):
-        step()
-    barrier(ws)
-    sampler = ClockSampler(local)
-    bj.launch_count_reset()
-    with sampler:
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    def timed(inverse=False):
+        for _ in range(args.warmup):
+            step(inverse=inverse)
         barrier(ws)
-        e0.record(stream)
-        for i in range(args.steps):
-            step(evs[i] if args.config == "C5" else None)
-        e1.record(stream)
-        barrier(ws)
-    launches = bj.launch_count()
+        sampler = ClockSampler(local)
+        bj.launch_count_reset()
+        with sampler:
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+            barrier(ws)
+            e0.record(stream)
+            for i in range(args.steps):
+                step(evs[i] if args.config == "C5" else None, inverse)
+            e1.record(stream)
+            barrier(ws)
+        return e0, e1, evs, bj.launch_count(), sampler
+
+    e0, e1, evs, launches, sampler = timed()
     t_ms = max_over_ranks(e0.elapsed_time(e1), ws)
     ms = t_ms / args.steps
+    inverse_variant = None
+    if args.config == "C5":
+        i0, i1, ievs, ilaunch, _ = timed(inverse=True)
+        ims = max_over_ranks(i0.elapsed_time(i1), ws) / args.steps
+        isetup = float(np.mean([e[0].elapsed_time(e[1]) for e in ievs]))
+        iapply = (ims - isetup) / napply
+        inv_bytes = int((8 * m * m + 16 * m + 16).sum().item())     # GEMV: Dinv + x in + y out + offsets
+        inverse_variant = {"ms_per_step": ims, "value": ws / (ims * 1e-3), "unit": "setups/s",
+                           "step": "bj_setup_inverse (extract + Gauss-Jordan inverses) + 100 bj_apply (GEMV)",
+                           "breakdown_ms": {"setup": isetup, "apply": iapply},
+                           "apply_roofline": {"achieved": inv_bytes / (iapply * 1e-3) / 1e9,
+                                              "frac": inv_bytes / (iapply * 1e-3) / 1e9 / load_peaks()[0],
+                                              "bytes": inv_bytes}, "gpu_launches": ilaunch}
     line = {"n_gpus": ws, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (counter-based FEM CSR generated on device)",
             "gpu_launches": launches, "clocks": sampler.summary()}
@@ -570,6 +591,7 @@ def run_fem(args, ws, rank, local):
                      "unit": "setups/s", "higher_is_better": True,
                      "config": {"workload": CONFIGS["C5"][4], "block": b, "rows_per_gpu": n, "applies": napply},
                      "breakdown_ms": {"setup": setup_ms, "apply": apply_ms},
+                     "inverse_variant": inverse_variant,
                      "step_hbm": {"algorithmic_bytes": ext_bytes + getrf_bytes + napply * getrs_bytes,
                                   "achieved_gbs": (ext_bytes + getrf_bytes + napply * getrs_bytes) / (ms * 1e-3) / 1e9},
                      "roofline": {"bound": "hbm", "kernel": "bj_apply", "achieved": getrs_bytes / (apply_ms * 1e-3) / 1e9,

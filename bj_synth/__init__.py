@@ -5,7 +5,8 @@ and builds input structures; both the oracle (tests, cpu baseline) and the
 CUDA path consume what it produces.  The device-side generator in
 ``paper_conf_icpp_anztdfq17_b200/csrc/synth.cu`` implements the *same*
 counter-based generator (splitmix64 keyed by (seed, global index)); the two
-are checked bit for bit against each other in ``tests/test_gpu_synth.py``.
+are checked bit for bit against each other in ``tests/test_gpu_parity.py``
+(test_device_generator_matches_host_generator) and ``tests/test_gpu_extract.py``.
 Because every value depends only on (seed, global index), any shard or
 subset of a workload regenerates identically.
 

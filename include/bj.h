@@ -195,6 +195,30 @@ bj_status bj_apply(bj_handle *handle, const void *x, void *y, bj_stream_t stream
 bj_status bj_destroy(bj_handle *handle);
 
 /* ---------------------------------------------------------------------------
+ * NEXT(3) -- inversion-based block-Jacobi: "explicitly
+ * compute the block-inverse before the iterative solution phase, and apply
+ * the preconditioner as a matrix-vector multiplication".
+ * bj_getri_vbatched: in place, blocks->values (packed per bj_layout) are
+ *   replaced by the inverses, column-major, computed by Gauss-Jordan
+ *   elimination with implicit partial pivoting (readings R23-R25 of DESIGN.md:
+ *   the GETRF pivot rule on the working matrix, IEEE division, single-rounding
+ *   FMA, unscaled pivot rows divided at the end).  pivots[vec_off[b] + k] =
+ *   pivot row of step k, info as for GETRF (k+1 for the first zero pivot; the
+ *   "inverse" of a singular block holds the IEEE results of the divisions by
+ *   zero; -1 for an order outside 0..32, block untouched).
+ * bj_gemv_vbatched: y_b = Dinv_b x_b per block (R26: fma chain over the
+ *   columns in order, from +0); x, y packed at inv->vec_off; y may alias x.
+ * bj_setup_inverse: like bj_setup with bj_getri_vbatched instead of GETRF;
+ *   bj_apply on such a handle runs bj_gemv_vbatched.
+ * ------------------------------------------------------------------------- */
+bj_status bj_getri_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info,
+                            const bj_plan *plan, bj_stream_t stream);
+bj_status bj_gemv_vbatched(const bj_batch *inv, const void *x, void *y,
+                           const bj_plan *plan, bj_stream_t stream);
+bj_status bj_setup_inverse(bj_handle *handle, const bj_csr *A, const int32_t *block_ptr,
+                           bj_batch *inverses, int32_t *pivots, int32_t *info, bj_stream_t stream);
+
+/* ---------------------------------------------------------------------------
  * Hot-path row a6 -- contiguous cost-balanced batch partitioner (multi-GPU;
  * not in the paper, which is single-GPU P:648).  HOST function.
  *   cost_b = m_b^2, P(i) = sum_{b<i} cost_b (int64),

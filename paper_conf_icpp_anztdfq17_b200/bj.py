@@ -25,6 +25,7 @@ _STATUS = {0: "BJ_OK", -1: "BJ_ERR_ARG", -2: "BJ_ERR_BLOCK_SIZE", -3: "BJ_ERR_AL
 EXPORTS = (
     "bj_status_string", "bj_version", "bj_layout", "bj_layout_from_block_ptr", "bj_plan_create",
     "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_gesv_vbatched",
+    "bj_getri_vbatched", "bj_gemv_vbatched", "bj_setup_inverse",
     "bj_create", "bj_setup",
     "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
     "bj_launch_count", "bj_launch_count_reset", "bj_supervariable_blocking",
@@ -70,6 +71,9 @@ def lib() -> ctypes.CDLL:
             "bj_getrf_vbatched": ([P, P, P, P, P], I32),
             "bj_getrs_vbatched": ([P, P, P, P, P, P], I32),
             "bj_gesv_vbatched": ([P, P, P, P, P, P, P], I32),
+            "bj_getri_vbatched": ([P, P, P, P, P], I32),
+            "bj_gemv_vbatched": ([P, P, P, P, P], I32),
+            "bj_setup_inverse": ([P, P, P, P, P, P, P], I32),
             "bj_create": ([P], I32),
             "bj_setup": ([P, P, P, P, P, P, P], I32),
             "bj_apply": ([P, P, P, P], I32),
@@ -227,6 +231,20 @@ def gesv(batch: Batch, pivots: torch.Tensor, info: torch.Tensor, rhs: torch.Tens
                                   plan.handle if plan else None, _stream(stream)), "bj_gesv_vbatched")
 
 
+def getri(batch: Batch, pivots: torch.Tensor, info: torch.Tensor, plan: Plan | None = None, stream=None):
+    """NEXT(3): in-place block inverses by Gauss-Jordan elimination (R23-R25)."""
+    b = batch.c()
+    _check(lib().bj_getri_vbatched(ctypes.byref(b), _p(pivots), _p(info), plan.handle if plan else None,
+                                   _stream(stream)), "bj_getri_vbatched")
+
+
+def gemv(inv: Batch, x: torch.Tensor, y: torch.Tensor, plan: Plan | None = None, stream=None):
+    """NEXT(3): y = Dinv x per block (R26); y may be x."""
+    b = inv.c()
+    _check(lib().bj_gemv_vbatched(ctypes.byref(b), _p(x), _p(y), plan.handle if plan else None, _stream(stream)),
+           "bj_gemv_vbatched")
+
+
 @dataclass
 class Csr:
     row_ptr: torch.Tensor     # int64[nrows+1]
@@ -263,6 +281,15 @@ class Handle:
         _check(lib().bj_setup(self._h, ctypes.byref(a), _p(block_ptr), ctypes.byref(f), _p(pivots), _p(info),
                               _stream(stream)), "bj_setup")
         self._keep = (A, block_ptr, factors, pivots, info)
+
+    def setup_inverse(self, A: Csr, block_ptr: torch.Tensor, inverses: Batch, pivots: torch.Tensor,
+                      info: torch.Tensor, stream=None):
+        """NEXT(3): setup = extract + explicit inverses (apply then = GEMV)."""
+        a = A.c()
+        f = inverses.c()
+        _check(lib().bj_setup_inverse(self._h, ctypes.byref(a), _p(block_ptr), ctypes.byref(f), _p(pivots),
+                                      _p(info), _stream(stream)), "bj_setup_inverse")
+        self._keep = (A, block_ptr, inverses, pivots, info)
 
     def apply(self, x: torch.Tensor, y: torch.Tensor, stream=None):
         _check(lib().bj_apply(self._h, _p(x), _p(y), _stream(stream)), "bj_apply")

@@ -51,6 +51,7 @@ struct bj_plan {
 
 struct bj_handle {
     bool ready = false;
+    bool inverse = false;              // NEXT(3): factors hold explicit inverses (apply = GEMV)
     bj_batch factors{};
     int32_t *pivots = nullptr;
     bj_plan plan;
@@ -257,6 +258,61 @@ bj_status bj_gesv_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, con
     return st;
 }
 
+bj_status bj_getri_vbatched(bj_batch *blocks, int32_t *pivots, int32_t *info, const bj_plan *plan,
+                            bj_stream_t stream) {
+    pool_keep_memory();
+    bj_status st = check_batch(blocks, true);
+    if (st != BJ_OK) return st;
+    if (blocks->nblocks > 0 && (!pivots || !info)) return BJ_ERR_ARG;
+    if (plan && plan->nblocks != blocks->nblocks) return BJ_ERR_ARG;
+    if (blocks->nblocks == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    bj_plan tmp;
+    const bj_plan *p = plan;
+    if (!p) {
+        if ((st = plan_alloc_build(&tmp, blocks->nblocks, blocks->sizes, s)) != BJ_OK) {
+            plan_free_async(&tmp, s);
+            return st;
+        }
+        p = &tmp;
+    }
+    if (blocks->dtype == BJ_F64)
+        st = getri_run<double>((double *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                               blocks->sizes, s);
+    else
+        st = getri_run<float>((float *)blocks->values, blocks->val_off, blocks->vec_off, pivots, info, p->view(),
+                              blocks->sizes, s);
+    if (!plan) plan_free_async(&tmp, s);
+    return st;
+}
+
+bj_status bj_gemv_vbatched(const bj_batch *inv, const void *x, void *y, const bj_plan *plan, bj_stream_t stream) {
+    pool_keep_memory();
+    bj_status st = check_batch(inv, true);
+    if (st != BJ_OK) return st;
+    if (inv->nblocks > 0 && (!x || !y)) return BJ_ERR_ARG;
+    if (plan && plan->nblocks != inv->nblocks) return BJ_ERR_ARG;
+    if (inv->nblocks == 0) return BJ_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    bj_plan tmp;
+    const bj_plan *p = plan;
+    if (!p) {
+        if ((st = plan_alloc_build(&tmp, inv->nblocks, inv->sizes, s)) != BJ_OK) {
+            plan_free_async(&tmp, s);
+            return st;
+        }
+        p = &tmp;
+    }
+    if (inv->dtype == BJ_F64)
+        st = gemv_run<double>((const double *)inv->values, inv->val_off, inv->vec_off, (const double *)x,
+                              (double *)y, p->view(), s);
+    else
+        st = gemv_run<float>((const float *)inv->values, inv->val_off, inv->vec_off, (const float *)x, (float *)y,
+                             p->view(), s);
+    if (!plan) plan_free_async(&tmp, s);
+    return st;
+}
+
 bj_status bj_create(bj_handle **handle) {
     if (!handle) return BJ_ERR_ARG;
     bj_handle *h = new (std::nothrow) bj_handle();
@@ -265,8 +321,8 @@ bj_status bj_create(bj_handle **handle) {
     return BJ_OK;
 }
 
-bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *factors, int32_t *pivots,
-                   int32_t *info, bj_stream_t stream) {
+static bj_status setup_common(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *factors,
+                              int32_t *pivots, int32_t *info, bj_stream_t stream, bool inverse) {
     pool_keep_memory();
     if (!h || !A || !block_ptr || !factors) return BJ_ERR_ARG;
     bj_status st = check_batch(factors, true);
@@ -282,18 +338,32 @@ bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_b
     if ((st = bj_extract(A, block_ptr, factors, stream)) != BJ_OK) return st;
     plan_free_async(&h->plan, s);
     if ((st = plan_alloc_build(&h->plan, nb, factors->sizes, s)) != BJ_OK) return st;
-    if ((st = bj_getrf_vbatched(factors, pivots, info, &h->plan, stream)) != BJ_OK) return st;
+    st = inverse ? bj_getri_vbatched(factors, pivots, info, &h->plan, stream)
+                 : bj_getrf_vbatched(factors, pivots, info, &h->plan, stream);
+    if (st != BJ_OK) return st;
     h->factors = *factors;
     h->pivots = pivots;
     h->nrows = A->nrows;
+    h->inverse = inverse;
     h->ready = true;
     return BJ_OK;
+}
+
+bj_status bj_setup(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *factors, int32_t *pivots,
+                   int32_t *info, bj_stream_t stream) {
+    return setup_common(h, A, block_ptr, factors, pivots, info, stream, false);
+}
+
+bj_status bj_setup_inverse(bj_handle *h, const bj_csr *A, const int32_t *block_ptr, bj_batch *inverses,
+                           int32_t *pivots, int32_t *info, bj_stream_t stream) {
+    return setup_common(h, A, block_ptr, inverses, pivots, info, stream, true);
 }
 
 bj_status bj_apply(bj_handle *h, const void *x, void *y, bj_stream_t stream) {
     pool_keep_memory();
     if (!h || !x || !y) return BJ_ERR_ARG;
     if (!h->ready) return BJ_ERR_STATE;
+    if (h->inverse) return bj_gemv_vbatched(&h->factors, x, y, &h->plan, stream);
     return bj_getrs_vbatched(&h->factors, h->pivots, x, y, &h->plan, stream);
 }
 

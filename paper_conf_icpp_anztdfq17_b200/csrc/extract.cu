@@ -196,20 +196,15 @@ template <typename R>
 bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, const int64_t *val_off, R *out,
                       cudaStream_t s) {
     if (nb == 0) return BJ_OK;
-    static int grid = 0, hgrid = 0;
-    if (grid == 0) {
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_extract_warp<R>, kExtractThreads, 0);
-        grid = (per_sm < 1 ? 1 : per_sm) * sm_count();
-        hgrid = 2 * sm_count();
-    }
+    const int grid = persistent_grid(k_extract_warp<R>, kExtractThreads);
+    const int hgrid = 2 * sm_count();
     int32_t *heavy = nullptr;
     unsigned long long *nheavy = nullptr;
     const size_t hbytes = sizeof(int32_t) * (size_t)nb;
-    char *scratch = nullptr;
-    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch, 16 + hbytes, s));
-    nheavy = reinterpret_cast<unsigned long long *>(scratch);
-    heavy = reinterpret_cast<int32_t *>(scratch + 16);
+    AsyncScratch scratch(s);
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch.p, 16 + hbytes, s));
+    nheavy = reinterpret_cast<unsigned long long *>(scratch.p);
+    heavy = reinterpret_cast<int32_t *>(scratch.p + 16);
     BJ_CUDA_TRY(cudaMemsetAsync(nheavy, 0, sizeof(unsigned long long), s));
     const R *vals = static_cast<const R *>(A.values);
     k_extract_warp<R><<<grid, kExtractThreads, 0, s>>>(A.row_ptr, A.col_idx, vals, A.col_offset, block_ptr, nb,
@@ -218,7 +213,6 @@ bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, con
     k_extract_heavy<R><<<hgrid, kHeavyThreads, 0, s>>>(A.row_ptr, A.col_idx, vals, A.col_offset, block_ptr,
                                                        val_off, out, heavy, nheavy);
     BJ_LAUNCH_CHECK();
-    BJ_CUDA_TRY(cudaFreeAsync(scratch, s));
     return BJ_OK;
 }
 

@@ -28,16 +28,10 @@ template <typename R, bool SOLVE>
 static bj_status getrf_solve_run(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
                                  const PlanView &p, const int32_t *sizes, const R *b, R *x, cudaStream_t s) {
     if (p.nblocks == 0) return BJ_OK;
-    char *scratch = nullptr;
-    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch, 16 + sizeof(int32_t) * (size_t)p.nblocks, s));
-    // the scratch is released (stream-ordered) on every return path
-    struct Free {
-        char *p;
-        cudaStream_t s;
-        ~Free() { cudaFreeAsync(p, s); }
-    } guard{scratch, s};
-    unsigned *safe_count = reinterpret_cast<unsigned *>(scratch);
-    int32_t *safe_list = reinterpret_cast<int32_t *>(scratch + 16);
+    AsyncScratch scratch(s);                 // released (stream-ordered) on every return path
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch.p, 16 + sizeof(int32_t) * (size_t)p.nblocks, s));
+    unsigned *safe_count = reinterpret_cast<unsigned *>(scratch.p);
+    int32_t *safe_list = reinterpret_cast<int32_t *>(scratch.p + 16);
     BJ_CUDA_TRY(cudaMemsetAsync(safe_count, 0, sizeof(unsigned), s));
     bj_status st;
     // orders 32..17: one kernel per order (each gets the register allocation of
@@ -55,6 +49,12 @@ static bj_status getrf_solve_run(R *A, const int64_t *val_off, const int64_t *ve
     k_getrf_safe<R><<<sm_count() * 2, 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info, safe_list, safe_count,
                                                    b, x);
     BJ_LAUNCH_CHECK();
+    k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
+    BJ_LAUNCH_CHECK();
+    return BJ_OK;
+}
+
+bj_status info_trivial_run(int32_t *info, const PlanView &p, cudaStream_t s) {
     k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
     BJ_LAUNCH_CHECK();
     return BJ_OK;

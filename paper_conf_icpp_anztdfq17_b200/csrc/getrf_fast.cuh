@@ -68,28 +68,6 @@ template <> __device__ __forceinline__ bool fast_ok<float>(float x) {
     return ((b & 0x7fffffffu) - (88u << 23) < (223u << 23) - (88u << 23)) || b == 0u;
 }
 
-// Per-tile max of a 32-bit key.  Full warp: one REDUX; 2 or 4 tiles: one
-// REDUX per tile (others contribute 0); smaller tiles: butterfly.
-template <int T>
-__device__ __forceinline__ unsigned tile_max_key(unsigned key, int t) {
-    if constexpr (T == 32) {
-        return __reduce_max_sync(kFull, key);
-    } else if constexpr (T >= 8) {
-        unsigned out = 0;
-#pragma unroll
-        for (int i = 0; i < 32 / T; ++i) {
-            const unsigned v = __reduce_max_sync(kFull, t == i ? key : 0u);
-            if (t == i) out = v;
-        }
-        return out;
-    } else {
-        unsigned v = key;
-#pragma unroll
-        for (int off = T / 2; off >= 1; off >>= 1) v = max(v, __shfl_xor_sync(kFull, v, off));
-        return v;
-    }
-}
-
 // Row stride of the panel buffer: fp64 34 elements (272 B = 17 x 16 B, an
 // odd number of 16-B units, so the STS.128 of the panel's pivot lanes hit
 // distinct bank groups)
@@ -701,22 +679,6 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
-// Launch grid per (kernel, device): resident CTAs per SM x SMs.
-template <typename K>
-int persistent_grid(K kernel, int threads) {
-    static int cached[64] = {0};
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev < 0 || dev >= 64) dev = 0;
-    if (cached[dev] == 0) {
-        int per_sm = 0;
-        cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0);
-        cached[dev] = (per_sm < 1 ? 1 : per_sm) * sm_count();
-    }
-    return cached[dev];
-}
-
 // Launch with programmatic stream serialization (PDL, see k_getrf_fast).
 template <typename R, int MLO, int MHI, bool SOLVE>
 bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
@@ -724,7 +686,7 @@ bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off
                             cudaStream_t s) {
     auto kern = k_getrf_fast<R, MLO, MHI, BJ_FAST_DEFAULT, SOLVE>;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(persistent_grid(kern, kFastThreads));
+    cfg.gridDim = dim3(persistent_grid(kern, kFastThreads, true));
     cfg.blockDim = dim3(kFastThreads);
     cfg.dynamicSmemBytes = 0;
     cfg.stream = s;

@@ -130,12 +130,7 @@ k_getrs_class(const R *__restrict__ LU, const int64_t *__restrict__ val_off, con
 template <typename R, int MLO, int MHI>
 bj_status launch_getrs_class(const R *LU, const int64_t *val_off, const int64_t *vec_off, const int32_t *piv,
                               const R *b, R *x, const PlanView &p, cudaStream_t s) {
-    static int grid = 0;
-    if (grid == 0) {
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_getrs_class<R, MLO, MHI>, kGetrsThreads, 0);
-        grid = (per_sm < 1 ? 1 : per_sm) * sm_count();
-    }
+    const int grid = persistent_grid(k_getrs_class<R, MLO, MHI>, kGetrsThreads);
     k_getrs_class<R, MLO, MHI><<<grid, kGetrsThreads, 0, s>>>(LU, val_off, vec_off, piv, b, x, p.order,
                                                                 p.bin_start);
     BJ_LAUNCH_CHECK();

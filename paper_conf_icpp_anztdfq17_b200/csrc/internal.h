@@ -26,6 +26,14 @@ bj_status getrf_run(R *values, const int64_t *val_off, const int64_t *vec_off, i
 template <typename R>
 bj_status gesv_run(R *values, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
                    const PlanView &plan, const int32_t *sizes, const R *b, R *x, cudaStream_t s);
+bj_status info_trivial_run(int32_t *info, const PlanView &plan, cudaStream_t s);
+// NEXT(3): inversion-based variant (getri.cu)
+template <typename R>
+bj_status getri_run(R *values, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
+                    const PlanView &plan, const int32_t *sizes, cudaStream_t s);
+template <typename R>
+bj_status gemv_run(const R *dinv, const int64_t *val_off, const int64_t *vec_off, const R *x, R *y,
+                   const PlanView &plan, cudaStream_t s);
 template <typename R>
 bj_status getrs_run(const R *lu, const int64_t *val_off, const int64_t *vec_off, const int32_t *piv,
                     const R *b, R *x, const PlanView &plan, cudaStream_t s);

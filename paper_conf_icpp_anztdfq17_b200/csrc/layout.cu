@@ -162,15 +162,15 @@ bj_status build_plan(int64_t nb, const int32_t *sizes, int32_t *order, int64_t *
         return BJ_OK;
     }
     const int64_t ntiles = (nb + kPlanTile - 1) / kPlanTile;
-    int64_t *hist = nullptr;
-    BJ_CUDA_TRY(cudaMallocAsync((void **)&hist, sizeof(int64_t) * kBins * ntiles, s));
+    AsyncScratch scratch(s);                 // released on every return path
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch.p, sizeof(int64_t) * kBins * ntiles, s));
+    int64_t *hist = reinterpret_cast<int64_t *>(scratch.p);
     k_plan_hist<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist);
     BJ_LAUNCH_CHECK();
     k_plan_offsets<<<1, 1024, 0, s>>>(hist, ntiles, bin_start);
     BJ_LAUNCH_CHECK();
     k_plan_scatter<<<(unsigned)ntiles, kPlanThreads, 0, s>>>(sizes, nb, hist, order);
     BJ_LAUNCH_CHECK();
-    BJ_CUDA_TRY(cudaFreeAsync(hist, s));
     return BJ_OK;
 }
 

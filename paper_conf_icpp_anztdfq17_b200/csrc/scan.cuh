@@ -104,15 +104,15 @@ template <class F>
 bj_status run_scan(F f, int64_t n, cudaStream_t s) {
     if (n == 0) return f.store_empty(s);
     const int64_t ntiles = (n + kScanTile - 1) / kScanTile;
-    I64x2 *partial = nullptr;
-    BJ_CUDA_TRY(cudaMallocAsync((void **)&partial, sizeof(I64x2) * ntiles, s));
+    AsyncScratch scratch(s);                 // released on every return path
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch.p, sizeof(I64x2) * ntiles, s));
+    I64x2 *partial = reinterpret_cast<I64x2 *>(scratch.p);
     k_scan_reduce<F><<<(unsigned)ntiles, kScanThreads, 0, s>>>(f, n, partial);
     BJ_LAUNCH_CHECK();
     k_scan_partials<<<1, kScanThreads, 0, s>>>(partial, ntiles);
     BJ_LAUNCH_CHECK();
     k_scan_down<F><<<(unsigned)ntiles, kScanThreads, 0, s>>>(f, n, partial);
     BJ_LAUNCH_CHECK();
-    BJ_CUDA_TRY(cudaFreeAsync(partial, s));
     return BJ_OK;
 }
 

@@ -1,6 +1,7 @@
 // synth.cu -- device-side seeded input generators (bench / test inputs only;
 // not part of the method).  Bit-identical to the host module bj_synth/ (the
-// same splitmix64 counter streams); checked in tests/test_gpu_synth.py.
+// same splitmix64 counter streams); checked in tests/test_gpu_parity.py
+// (test_device_generator_matches_host_generator) and tests/test_gpu_extract.py.
 #include "bj_synth.h"
 #include "scan.cuh"
 

@@ -3,7 +3,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <vector>
-#include "getrf_pair.cuh"
+#include "../../scripts/micro/getrf_pair.cuh"
 
 namespace bj {
 void count_launch(int) {}
