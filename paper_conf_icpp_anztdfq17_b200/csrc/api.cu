@@ -335,11 +335,19 @@ static bj_status setup_common(bj_handle *h, const bj_csr *A, const int32_t *bloc
     h->ready = false;
     if ((st = layout_block_ptr(nb, block_ptr, es, factors->sizes, factors->vec_off, factors->val_off, s)) != BJ_OK)
         return st;
-    if ((st = bj_extract(A, block_ptr, factors, stream)) != BJ_OK) return st;
+    if (A->nrows < 0 || A->nnz < 0 || !A->row_ptr || (A->nnz > 0 && (!A->col_idx || !A->values))) return BJ_ERR_ARG;
     plan_free_async(&h->plan, s);
     if ((st = plan_alloc_build(&h->plan, nb, factors->sizes, s)) != BJ_OK) return st;
-    st = inverse ? bj_getri_vbatched(factors, pivots, info, &h->plan, stream)
-                 : bj_getrf_vbatched(factors, pivots, info, &h->plan, stream);
+    if (inverse) {
+        if ((st = bj_extract(A, block_ptr, factors, stream)) != BJ_OK) return st;
+        st = bj_getri_vbatched(factors, pivots, info, &h->plan, stream);
+    } else if (factors->dtype == BJ_F64) {          // NEXT(1): extraction fused into GETRF
+        st = setup_run<double>(*A, block_ptr, (double *)factors->values, factors->val_off, factors->vec_off,
+                               pivots, info, h->plan.view(), factors->sizes, s);
+    } else {
+        st = setup_run<float>(*A, block_ptr, (float *)factors->values, factors->val_off, factors->vec_off,
+                              pivots, info, h->plan.view(), factors->sizes, s);
+    }
     if (st != BJ_OK) return st;
     h->factors = *factors;
     h->pivots = pivots;

@@ -15,15 +15,13 @@
 //  * persistent grid, blocks taken in row order (streaming CSR reads).
 #include "common.cuh"
 #include "internal.h"
-
-#include <climits>
+#include "extract_tile.cuh"
 
 namespace bj {
 
 constexpr int kExtractWarps = 4;
 constexpr int kExtractThreads = 32 * kExtractWarps;
 constexpr int kHeavyThreads = 256;
-constexpr int64_t kHeavy = 8192;     // stored entries per block above which the CTA path is used
 
 template <typename R>
 __device__ __forceinline__ void write_tile(R *__restrict__ dst, const R *src, int nelem_padded) {
@@ -34,12 +32,14 @@ __device__ __forceinline__ void write_tile(R *__restrict__ dst, const R *src, in
     for (int i = threadIdx.x & 31; i < n16; i += 32) d4[i] = s4[i];
 }
 
+// mlo_skip: blocks of order >= mlo_skip (and at most kHeavy entries) are left
+// to the fused setup kernel (0 = extract every block).
 template <typename R>
 __global__ void __launch_bounds__(kExtractThreads)
 k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col_idx,
                const R *__restrict__ values, int64_t col_offset, const int32_t *__restrict__ block_ptr,
                int64_t nb, const int64_t *__restrict__ val_off, R *__restrict__ out,
-               int32_t *__restrict__ heavy, unsigned long long *__restrict__ nheavy) {
+               int32_t *__restrict__ heavy, unsigned long long *__restrict__ nheavy, int mlo_skip) {
     __shared__ __align__(16) R tile[kExtractWarps][kMaxM * kMaxM];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     R *T = tile[w];
@@ -77,77 +77,10 @@ k_extract_warp(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ 
             if (lane == 0) heavy[atomicAdd(nheavy, 1ull)] = (int32_t)b;
             continue;
         }
+        if (mlo_skip > 0 && m >= mlo_skip) continue;           // the fused setup extracts it
         const int q = 16 / (int)sizeof(R);
         const int np = (m * m + q - 1) / q * q;
-        for (int i = lane; i < np; i += 32) T[i] = R(0);
-        __syncwarp();
-        const int64_t cb = (int64_t)bs + col_offset, ce = (int64_t)be + col_offset;
-        // The block's rows are one contiguous entry range [e0, e1): the warp
-        // scans it in 32-entry chunks (coalesced col-indices),
-        // kU chunks per round so kU loads per lane are in flight, and the
-        // value loads of one round overlap the col-index loads of the next.
-        // Row of entry e: rows starting at or before the chunk start (ballot)
-        // plus row starts inside the chunk at or before e (one REDUX.OR mask).
-        const int rel = lane < m ? (int)(rpv - e0) : INT_MAX;   // row start, relative
-        const int len = (int)(e1 - e0);
-        // The row-start mask counts each start position once, so a block with
-        // an empty row (two rows starting at the same entry) takes the plain
-        // row-by-row scan instead (rare: FEM-like matrices have none).
-        const int rel_next = __shfl_down_sync(kFull, rel, 1);
-        const bool has_empty = __any_sync(kFull, lane < m && (lane + 1 < m ? rel_next == rel : rel == len));
-        if (has_empty) {
-            for (int r = 0; r < m; ++r) {
-                const int rs = __shfl_sync(kFull, rel, r);
-                const int re = r + 1 < m ? __shfl_sync(kFull, rel, r + 1) : len;
-                for (int e = rs + lane; e < re; e += 32) {
-                    const int64_t c = __ldg(col_idx + e0 + e);
-                    if (c >= cb && c < ce) T[r + (int)(c - cb) * m] = __ldg(values + e0 + e);
-                }
-            }
-        } else {
-            const int nch = (len + 31) >> 5;
-            constexpr int kU = 8;
-            int32_t cc[kU];
-            auto load_cols = [&](int c0) {
-#pragma unroll
-                for (int u = 0; u < kU; ++u) {
-                    const int e = ((c0 + u) << 5) + lane;
-                    cc[u] = e < len ? __ldg(col_idx + e0 + e) : -1;
-                }
-            };
-            load_cols(0);
-            for (int c0 = 0; c0 < nch; c0 += kU) {
-                int32_t cv[kU];
-#pragma unroll
-                for (int u = 0; u < kU; ++u) cv[u] = cc[u];
-                if (c0 + kU < nch) load_cols(c0 + kU);
-                // all value loads of the round first (in-order issue: a store that
-                // waits on its load would otherwise serialise the chunks), then
-                // the scatter into the smem tile
-                R vv[kU];
-                int at[kU];
-#pragma unroll
-                for (int u = 0; u < kU; ++u) {
-                    const int E = (c0 + u) << 5;
-                    at[u] = -1;
-                    if (E < len) {                                        // warp-uniform
-                        const int row0 = __popc(__ballot_sync(kFull, rel <= E)) - 1;
-                        const unsigned starts =
-                            __reduce_or_sync(kFull, (rel > E && rel < E + 32) ? 1u << (rel - E) : 0u);
-                        const int row = row0 + __popc(starts & ((2u << lane) - 1u));
-                        const int64_t c = cv[u];
-                        if (c >= cb && c < ce) {
-                            at[u] = row + (int)(c - cb) * m;
-                            vv[u] = __ldg(values + e0 + E + lane);
-                        }
-                    }
-                }
-#pragma unroll
-                for (int u = 0; u < kU; ++u)
-                    if (at[u] >= 0) T[at[u]] = vv[u];
-            }
-        }
-        __syncwarp();
+        extract_block_warp<R>(col_idx, values, col_offset, bs, m, rpv, e0, e1, T);
         write_tile(out + __ldg(val_off + b), T, np);
         __syncwarp();
     }
@@ -194,7 +127,7 @@ k_extract_heavy(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__
 
 template <typename R>
 bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, const int64_t *val_off, R *out,
-                      cudaStream_t s) {
+                      cudaStream_t s, int mlo_skip) {
     if (nb == 0) return BJ_OK;
     const int grid = persistent_grid(k_extract_warp<R>, kExtractThreads);
     const int hgrid = 2 * sm_count();
@@ -208,7 +141,7 @@ bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, con
     BJ_CUDA_TRY(cudaMemsetAsync(nheavy, 0, sizeof(unsigned long long), s));
     const R *vals = static_cast<const R *>(A.values);
     k_extract_warp<R><<<grid, kExtractThreads, 0, s>>>(A.row_ptr, A.col_idx, vals, A.col_offset, block_ptr, nb,
-                                                       val_off, out, heavy, nheavy);
+                                                       val_off, out, heavy, nheavy, mlo_skip);
     BJ_LAUNCH_CHECK();
     k_extract_heavy<R><<<hgrid, kHeavyThreads, 0, s>>>(A.row_ptr, A.col_idx, vals, A.col_offset, block_ptr,
                                                        val_off, out, heavy, nheavy);
@@ -217,8 +150,8 @@ bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, con
 }
 
 template bj_status extract_run<double>(const bj_csr &, const int32_t *, int64_t, const int64_t *, double *,
-                                       cudaStream_t);
+                                       cudaStream_t, int);
 template bj_status extract_run<float>(const bj_csr &, const int32_t *, int64_t, const int64_t *, float *,
-                                      cudaStream_t);
+                                      cudaStream_t, int);
 
 }  // namespace bj

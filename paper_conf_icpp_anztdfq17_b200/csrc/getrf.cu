@@ -60,6 +60,54 @@ bj_status info_trivial_run(int32_t *info, const PlanView &p, cudaStream_t s) {
     return BJ_OK;
 }
 
+template <typename R, int M>
+bj_status launch_setup_fused(const bj_csr &Acsr, const int32_t *block_ptr, R *A, const int64_t *val_off,
+                             const int64_t *vec_off, int32_t *piv, int32_t *info, const PlanView &p,
+                             int32_t *safe_list, unsigned *safe_count, cudaStream_t s);
+
+// NEXT(1): setup = extraction of the blocks of order <= 16 (and of blocks
+// with more than kHeavy entries) into `out`, then the fused extract + GETRF
+// kernels for orders 32..17 (no dense round trip through HBM), then the
+// GETRF classes 1-16 and the safe path -- outputs bit-identical to
+// extract_run + getrf_run.
+template <typename R>
+bj_status setup_run(const bj_csr &Acsr, const int32_t *block_ptr, R *A, const int64_t *val_off,
+                    const int64_t *vec_off, int32_t *piv, int32_t *info, const PlanView &p, const int32_t *sizes,
+                    cudaStream_t s) {
+    if (p.nblocks == 0) return BJ_OK;
+    bj_status st;
+    if ((st = extract_run<R>(Acsr, block_ptr, p.nblocks, val_off, A, s, 17)) != BJ_OK) return st;
+    AsyncScratch scratch(s);
+    BJ_CUDA_TRY(cudaMallocAsync((void **)&scratch.p, 16 + sizeof(int32_t) * (size_t)p.nblocks, s));
+    unsigned *safe_count = reinterpret_cast<unsigned *>(scratch.p);
+    int32_t *safe_list = reinterpret_cast<int32_t *>(scratch.p + 16);
+    BJ_CUDA_TRY(cudaMemsetAsync(safe_count, 0, sizeof(unsigned), s));
+#define BJ_FUSED_M(M)                                                                                      \
+    if ((st = launch_setup_fused<R, M>(Acsr, block_ptr, A, val_off, vec_off, piv, info, p, safe_list,       \
+                                       safe_count, s)) != BJ_OK)                                           \
+        return st;
+    BJ_FUSED_M(32) BJ_FUSED_M(31) BJ_FUSED_M(30) BJ_FUSED_M(29) BJ_FUSED_M(28) BJ_FUSED_M(27) BJ_FUSED_M(26)
+    BJ_FUSED_M(25) BJ_FUSED_M(24) BJ_FUSED_M(23) BJ_FUSED_M(22) BJ_FUSED_M(21) BJ_FUSED_M(20) BJ_FUSED_M(19)
+    BJ_FUSED_M(18) BJ_FUSED_M(17)
+#undef BJ_FUSED_M
+#define BJ_GETRF_C(LO, HI)                                                                                  \
+    if ((st = launch_getrf_fast<R, LO, HI, false>(A, val_off, vec_off, piv, info, p, safe_list, safe_count,  \
+                                                  nullptr, nullptr, s)) != BJ_OK)                            \
+        return st;
+    BJ_GETRF_C(9, 16) BJ_GETRF_C(5, 8) BJ_GETRF_C(1, 4)
+#undef BJ_GETRF_C
+    k_getrf_safe<R><<<sm_count() * 2, 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info, safe_list, safe_count);
+    BJ_LAUNCH_CHECK();
+    k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
+    BJ_LAUNCH_CHECK();
+    return BJ_OK;
+}
+
+template bj_status setup_run<double>(const bj_csr &, const int32_t *, double *, const int64_t *, const int64_t *,
+                                     int32_t *, int32_t *, const PlanView &, const int32_t *, cudaStream_t);
+template bj_status setup_run<float>(const bj_csr &, const int32_t *, float *, const int64_t *, const int64_t *,
+                                    int32_t *, int32_t *, const PlanView &, const int32_t *, cudaStream_t);
+
 template <typename R>
 bj_status getrf_run(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
                     const PlanView &p, const int32_t *sizes, cudaStream_t s) {

@@ -269,6 +269,16 @@ __device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, int &inf, b
     });
 }
 
+// Fused setup (setup_fused.cuh): a block sent to the safe kernel must be in
+// memory, but the fused path extracted it into shared memory only; the tile
+// writes its original (S, column-major, ld M) to A first.
+template <typename R, int M>
+__device__ __forceinline__ void fused_spill(R *Ab, const R *S, bool tile_ok, int r, int T) {
+    if (tile_ok)
+        for (int i = r; i < M * M; i += T) Ab[i] = S[i];
+    __syncwarp();
+}
+
 // Fused GETRS (bj_gesv_vbatched): the factors are still in registers -- lane
 // r holds row r of the block, which is row pos = tag-1 of L\U -- so the solve
 // of P:218-238 (b := P b, eager unit-lower solve, eager upper solve with
@@ -306,7 +316,7 @@ __device__ __forceinline__ void getrf_tile_solve(const R (&a)[M], int pos, bool 
 // S: this tile's block staged in shared memory by the bulk copy (column-major,
 // leading dimension M); `after_load` runs once the block is in registers
 // (it re-arms the warp's staging buffer with the next task).
-template <typename R, int M, int F, bool SOLVE, class AfterLoad>
+template <typename R, int M, int F, bool SOLVE, class AfterLoad, bool FUSED = false>
 __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &tk, const R *S,
                                                 int32_t *__restrict__ piv, int32_t *__restrict__ info,
                                                 int32_t *__restrict__ safe_list, unsigned *__restrict__ safe_count,
@@ -332,6 +342,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     after_load();
     // Tiles with an entry outside the fast path's precondition go to the safe kernel.
     if (tile_bits<T>(__ballot_sync(kFull, !ok), tbase) != 0u) {
+        if constexpr (FUSED) fused_spill<R, M>(Ab, S, tile_ok, r, T);
         if (tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
         tile_ok = false;
     }
@@ -463,6 +474,9 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     // input; the other tiles of the warp go on (the solve's shuffles need
     // every lane, so no lane returns early).
     const bool again = tile_bits<T>(__ballot_sync(kFull, redo && tile_ok), tbase) != 0u;
+    if constexpr (FUSED) {
+        if (again) fused_spill<R, M>(Ab, S, tile_ok, r, T);
+    }
     if (again && tile_ok && r == 0) safe_list[atomicAdd(safe_count, 1u)] = blk;
     const bool keep = tile_ok && !again;
     const bool row_keep = keep && (r < M);

@@ -39,9 +39,17 @@ bj_status getrs_run(const R *lu, const int64_t *val_off, const int64_t *vec_off,
                     const R *b, R *x, const PlanView &plan, cudaStream_t s);
 
 // a2
+// mlo_skip > 0: blocks of order >= mlo_skip with at most kHeavy entries are
+// left to the fused setup (setup_run)
 template <typename R>
 bj_status extract_run(const bj_csr &A, const int32_t *block_ptr, int64_t nb, const int64_t *val_off,
-                      R *out, cudaStream_t s);
+                      R *out, cudaStream_t s, int mlo_skip = 0);
+// NEXT(1): block-Jacobi setup with the extraction fused into GETRF for orders
+// 17..32 (setup_fused.cuh); the values of out must be laid out per block_ptr
+template <typename R>
+bj_status setup_run(const bj_csr &A, const int32_t *block_ptr, R *out, const int64_t *val_off,
+                    const int64_t *vec_off, int32_t *piv, int32_t *info, const PlanView &plan,
+                    const int32_t *sizes, cudaStream_t s);
 
 // NEXT(2)
 bj_status supervariable_run(const bj_csr &A, int32_t bound, int32_t *block_ptr, int64_t *nblocks_h,

@@ -220,3 +220,74 @@ def test_block_jacobi_block_ptr_offset():
     yo = oracle.getrs_batch(sz, vl, vo, LU, po, x.cpu().numpy())
     assert np.array_equal(info.cpu().numpy(), io) and np.array_equal(piv.cpu().numpy(), po)
     assert np.array_equal(bits(y.cpu().numpy()), bits(yo))
+
+
+def _setup_vs_separate(A, bp, n, dtype):
+    """bj_setup (NEXT(1): extraction fused into GETRF for orders 17..32) equals
+    bj_extract + bj_getrf_vbatched bit for bit (factors, pivots, info)."""
+    bpt = torch.from_numpy(np.ascontiguousarray(bp, dtype=np.int32)).cuda()
+    sizes, vec, val = bj.layout_from_block_ptr(bpt, dtype)
+    nb = len(bp) - 1
+    rows = int(bp[-1] - bp[0])
+    fac = bj.Batch(sizes, vec, val, torch.full((int(val[-1].item()),), 7.0, dtype=dtype, device="cuda"))
+    piv = torch.full((rows,), -5, dtype=torch.int32, device="cuda")
+    info = torch.full((nb,), -9, dtype=torch.int32, device="cuda")
+    h = bj.Handle()
+    h.setup(A, bpt, fac, piv, info)
+    sep = bj.Batch(sizes, vec, val, torch.full_like(fac.values, 7.0))
+    bj.extract(A, bpt, sep)
+    piv2 = torch.full_like(piv, -5)
+    info2 = torch.full_like(info, -9)
+    bj.getrf(sep, piv2, info2)
+    torch.cuda.synchronize()
+    assert torch.equal(info, info2) and torch.equal(piv, piv2)
+    v = val.cpu().numpy()
+    m = sizes.cpu().numpy().astype(np.int64)
+    idx = np.concatenate([np.arange(v[i], v[i] + m[i] * m[i]) for i in range(nb)]) if nb else np.zeros(0, np.int64)
+    it = torch.from_numpy(idx).cuda()
+    a, b = fac.values[it], sep.values[it]
+    iv = torch.int64 if dtype == torch.float64 else torch.int32
+    assert torch.equal(a.view(iv), b.view(iv))
+    return fac, piv, info
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_fused_setup_mixed_orders_and_hubs(dtype):
+    """Block sizes 1..32 (fused for 17..32, separate below), hub rows (blocks
+    above kHeavy entries take the extract_heavy + safe path), random values
+    with pivoting; also checked against the oracle."""
+    rng = np.random.default_rng(31)
+    n = 20000
+    rows = []
+    for r in range(n):
+        if r in (40, 9000):
+            c = rng.choice(n, size=12000, replace=False)
+        else:
+            c = np.unique(np.clip(r + rng.integers(-25, 26, size=20), 0, n - 1))
+        rows.append(rng.permutation(c))
+    rp = np.concatenate([[0], np.cumsum([len(c) for c in rows])]).astype(np.int64)
+    ci = np.concatenate(rows).astype(np.int32)
+    va = rng.uniform(-1, 1, size=len(ci)).astype(NP[dtype])
+    cuts = [0]
+    while cuts[-1] < n:
+        cuts.append(min(n, cuts[-1] + int(rng.integers(1, 33))))
+    bp = np.array(cuts, np.int32)
+    A = bj.Csr(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), torch.from_numpy(va).cuda())
+    fac, piv, info = _setup_vs_separate(A, bp, n, dtype)
+    D, sz, vo, vl = oracle.extract(rp, ci, va, bp)
+    LU, po, io = oracle.getrf_batch(sz, vl, vo, D)
+    assert np.array_equal(info.cpu().numpy(), io) and np.array_equal(piv.cpu().numpy(), po)
+    got = fac.values.cpu().numpy()
+    for i in range(len(sz)):
+        mm = int(sz[i])
+        assert np.array_equal(bits(got[vl[i]: vl[i] + mm * mm]), bits(LU[vl[i]: vl[i] + mm * mm]))
+
+
+def test_fused_setup_c5_size():
+    """C5's per-GPU slab (1,998,216 rows, b = 24) in the bench's launch
+    configuration: fused setup == extract + getrf, bit for bit."""
+    nx, ny, nz = 174, 174, 22
+    n = 3 * nx * ny * nz
+    A = bj.synth_fem(nx, ny, nz, 0, n)
+    bp = S.uniform_block_ptr(n, 24)
+    _setup_vs_separate(A, bp, n, torch.float64)
