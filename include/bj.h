@@ -249,6 +249,19 @@ bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t 
                                     int64_t *nblocks_h, bj_stream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * Test hook (not the hot path), SYNCHRONOUS: checks on the device that the
+ * split IEEE divisions the kernels use for every quotient (R3) reproduce the
+ * correctly rounded quotient (__ddiv_rn / __fdiv_rn) on n pseudo-random
+ * operand pairs covering every exponent and the specials.  counts_h (HOST,
+ * 6 entries): [0] full division mismatches, [1] mismatches of the flag-only
+ * quotient where it claims validity, [2] its flagged count, [3] / [4] the
+ * same for the normal-divisor variant, [5] pairs tested.  sample_h (HOST,
+ * 3*nsample elements of dtype) receives (a, b, a/b) of the first pairs.
+ * ------------------------------------------------------------------------- */
+bj_status bj_selftest_div(bj_dtype dtype, int64_t n, uint64_t seed, uint64_t *counts_h, void *sample_h,
+                          int64_t nsample);
+
+/* ---------------------------------------------------------------------------
  * End-to-end call with HOST buffers (synchronous): copies sizes_h (nblocks),
  * blocks_h (nvalues elements, packed per bj_layout) and b_h (nvec elements)
  * to the device, runs layout + plan + GETRF + GETRS, and copies x_h (nvec),

@@ -25,7 +25,7 @@ _STATUS = {0: "BJ_OK", -1: "BJ_ERR_ARG", -2: "BJ_ERR_BLOCK_SIZE", -3: "BJ_ERR_AL
 EXPORTS = (
     "bj_status_string", "bj_version", "bj_layout", "bj_layout_from_block_ptr", "bj_plan_create",
     "bj_plan_destroy", "bj_extract", "bj_getrf_vbatched", "bj_getrs_vbatched", "bj_gesv_vbatched",
-    "bj_getri_vbatched", "bj_gemv_vbatched", "bj_setup_inverse",
+    "bj_getri_vbatched", "bj_gemv_vbatched", "bj_setup_inverse", "bj_selftest_div",
     "bj_create", "bj_setup",
     "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
     "bj_launch_count", "bj_launch_count_reset", "bj_supervariable_blocking",
@@ -74,6 +74,7 @@ def lib() -> ctypes.CDLL:
             "bj_getri_vbatched": ([P, P, P, P, P], I32),
             "bj_gemv_vbatched": ([P, P, P, P, P], I32),
             "bj_setup_inverse": ([P, P, P, P, P, P, P], I32),
+            "bj_selftest_div": ([I32, I64, ctypes.c_uint64, P, P, I64], I32),
             "bj_create": ([P], I32),
             "bj_setup": ([P, P, P, P, P, P, P], I32),
             "bj_apply": ([P, P, P, P], I32),
@@ -387,3 +388,14 @@ def synth_fem(nx: int, ny: int, nz: int, r0: int, r1: int, dtype=torch.float64, 
     _check(lib().bj_synth_fem_fill(nx, ny, nz, int(skew), r0, r1, _p(rp), _p(ci), _p(va), dtype_code(dtype),
                                    _stream(stream)), "bj_synth_fem_fill")
     return Csr(rp, ci[:nnz], va[:nnz], r0)
+
+
+def selftest_div(dtype: torch.dtype, n: int, seed: int = 1, nsample: int = 0):
+    """Test hook: device check of the split IEEE divisions (bj_selftest_div).
+    Returns (counts[6], sample (nsample, 3) array of a, b, a/b)."""
+    counts = np.zeros(6, dtype=np.uint64)
+    npdt = np.float64 if dtype == torch.float64 else np.float32
+    sample = np.zeros((max(nsample, 1), 3), dtype=npdt)
+    _check(lib().bj_selftest_div(dtype_code(dtype), int(n), int(seed), counts.ctypes.data_as(ctypes.c_void_p),
+                                 sample.ctypes.data_as(ctypes.c_void_p), int(nsample)), "bj_selftest_div")
+    return counts, sample[:nsample]
