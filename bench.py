@@ -301,7 +301,7 @@ def run_ours(args, ws, rank, local):
     getrf_bytes, getrs_bytes = algorithmic_bytes(my_sizes, dt)
 
     base = bj.new_batch(sizes, dt)
-    bj.synth_blocks(base, first=first)
+    bj.synth_blocks(base, first=first, kind=1 if args.kind == "int" else 0)
     rhs = bj.synth_rhs(base, first=first)
     nvec = int(base.vec_off[-1].item())
     piv = torch.empty(max(nvec, 1), dtype=torch.int32, device="cuda")
@@ -448,6 +448,7 @@ def run_ours(args, ws, rank, local):
             "scaling": scaling, "vs_baseline": None, "dtype": "f64" if dt == torch.float64 else "f32",
             "data": "synthetic (counter-based splitmix64, generated on device)",
             "config": {"workload": desc, "nblocks_total": nb_total, "nblocks_rank0": nb, "sizes": f"U{{{lo}..{hi}}}",
+                       "values": "U[-1,1)" if args.kind == "uniform" else "U{-3..3} integers (ties, singular blocks)",
                        "step": "layout + plan + bj_getrf_vbatched + bj_getrs_vbatched",
                        "parallelism": f"dp{ws} (contiguous cost-balanced shards, {scaling} scaling)",
                        "l2": f"inputs larger than L2: each step factors its own pristine {copy_bytes / 1e9:.2f} GB copy"},
@@ -629,6 +630,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-fused", action="store_true", help="skip the extra fused bj_gesv_vbatched measurement")
+    ap.add_argument("--kind", default="uniform", choices=["uniform", "int"],
+                    help="block values: U[-1,1) (default) or the tie-heavy integer stress set U{-3..3}")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
                     help="multi-GPU batched configs: shard the config's batch (strong) or replicate it per GPU (weak)")

@@ -46,8 +46,8 @@ static bj_status getrf_solve_run(R *A, const int64_t *val_off, const int64_t *ve
     BJ_GETRF_C(22, 22) BJ_GETRF_C(21, 21) BJ_GETRF_C(20, 20) BJ_GETRF_C(19, 19) BJ_GETRF_C(18, 18)
     BJ_GETRF_C(17, 17) BJ_GETRF_C(9, 16) BJ_GETRF_C(5, 8) BJ_GETRF_C(1, 4)
 #undef BJ_GETRF_C
-    k_getrf_safe<R><<<sm_count() * 2, 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info, safe_list, safe_count,
-                                                   b, x);
+    k_getrf_safe<R><<<persistent_grid(k_getrf_safe<R>, 128), 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info,
+                                                                           safe_list, safe_count, b, x);
     BJ_LAUNCH_CHECK();
     k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
     BJ_LAUNCH_CHECK();
@@ -96,7 +96,8 @@ bj_status setup_run(const bj_csr &Acsr, const int32_t *block_ptr, R *A, const in
         return st;
     BJ_GETRF_C(9, 16) BJ_GETRF_C(5, 8) BJ_GETRF_C(1, 4)
 #undef BJ_GETRF_C
-    k_getrf_safe<R><<<sm_count() * 2, 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info, safe_list, safe_count);
+    k_getrf_safe<R><<<persistent_grid(k_getrf_safe<R>, 128), 128, 0, s>>>(A, sizes, val_off, vec_off, piv, info,
+                                                                           safe_list, safe_count);
     BJ_LAUNCH_CHECK();
     k_info_trivial<<<sm_count(), 256, 0, s>>>(info, p.order, p.bin_start);
     BJ_LAUNCH_CHECK();

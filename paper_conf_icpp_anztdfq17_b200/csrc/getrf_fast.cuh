@@ -39,7 +39,8 @@
 //        writes only column k (never touched again) and a GER result is -0
 //        only through underflow.  Underflow is excluded by magnitudes: if
 //        every input and every final L\U entry is 0 or in [2^-450, 2^990)
-//        (fp32: [2^-39, 2^96)), every product l*u is 0 or >= 2^-900, a
+//        (fp32: [2^-39, 2^96); -0 allowed in the L part, which GER never
+//        touches after SCAL), every product l*u is 0 or >= 2^-900, a
 //        result below it in magnitude cannot cancel further, and every
 //        nonzero intermediate stays >= 2^-1006 (fp32 2^-126), above the
 //        subnormal range.  Blocks failing the input test go to k_getrf_safe
@@ -467,8 +468,13 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
             __syncwarp();
         }
     });
-    // Output test of the zero-multiplier argument (header comment).
-    static_for<0, M>([&](auto jc) { redo = redo || !fast_ok(a[decltype(jc)::value]); });
+    // Output test of the zero-multiplier argument (header comment).  The L part
+    // (columns < pos) may hold -0 (SCAL of a +0 entry by a negative pivot):
+    // GER never touches a column after its SCAL, so those zeros are final.
+    static_for<0, M>([&](auto jc) {
+        constexpr int j = decltype(jc)::value;
+        redo = redo || !(fast_ok(a[j]) || (a[j] == R(0) && j < tag - 1));
+    });
     // Tiles that hit a pivot ambiguity, a slow-path quotient or a failed
     // output test are redone by the safe kernel from the (still untouched)
     // input; the other tiles of the warp go on (the solve's shuffles need
@@ -743,22 +749,18 @@ k_getrf_safe(R *A, const int32_t *__restrict__ sizes, const int64_t *__restrict_
         int inf = 0;
         for (int k = 0; k < m; ++k) {
             const R v = r < m ? s[r + k * 33] : R(0);
-            unsigned long long key = 0ull;
-            if (tag == 0) {
-                key = (sizeof(R) == 8) ? ((unsigned long long)__double_as_longlong((double)v) & 0x7fffffffffffffffULL)
-                                       : (unsigned long long)(__float_as_uint((float)v) & 0x7fffffffu);
-                key += 1ull;
-            }
-            unsigned long long best = key;
-            int bl = r;
-#pragma unroll
-            for (int off = 16; off >= 1; off >>= 1) {
-                const unsigned long long ok = __shfl_xor_sync(kFull, best, off);
-                const int ol = __shfl_xor_sync(kFull, bl, off);
-                if (ok > best || (ok == best && ol < bl)) { best = ok; bl = ol; }
-            }
-            const int ipiv = bl;
-            const bool sing = (best == 1ull);
+            // exact key (R2) by three warp reductions: the largest high word
+            // of |v| among candidates (+1 so a zero candidate beats a
+            // non-candidate), the largest low word among those, the lowest
+            // lane among the maxima (R1)
+            const bool cand = (tag == 0);
+            const unsigned khi = cand ? Num<R>::key_hi(v) + 1u : 0u;
+            const unsigned mhi = __reduce_max_sync(kFull, khi);
+            const unsigned klo = (cand && khi == mhi) ? Num<R>::key_lo(v) : 0u;
+            const unsigned mlo = __reduce_max_sync(kFull, klo);
+            const unsigned who = (cand && khi == mhi && klo == mlo) ? (unsigned)r : 31u;
+            const int ipiv = (int)__reduce_min_sync(kFull, who);
+            const bool sing = (mhi == 1u) && (mlo == 0u);
             if (r == ipiv) tag = k + 1;
             const R d = s[ipiv + k * 33];
             if (!sing && tag == 0) {
