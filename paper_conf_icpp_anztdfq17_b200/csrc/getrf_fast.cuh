@@ -92,8 +92,9 @@ struct FastSmem {
 //   kPanel2/3/4 -- full-warp tiles: W-step panels (see getrf_w32_steps).
 //   kMin5 / kMin6 -- 5 / 6 CTAs (20 / 24 warps) per SM (102 / 85 registers).
 //   kMin4 -- 4 CTAs (16 warps) per SM (128 registers).
+//   kNoinline -- per-order tiles out of line (one launch per order range).
 constexpr int kPre = 1, kMin3 = 2, kVol = 4, kPanel2 = 8, kPanel3 = 16, kPanel4 = 32, kMin5 = 64, kMin6 = 128,
-              kMin4 = 256;
+              kMin4 = 256, kNoinline = 512;
 __host__ __device__ constexpr int panel_width(int F) {
     return (F & kPanel4) ? 4 : (F & kPanel3) ? 3 : (F & kPanel2) ? 2 : 1;
 }
@@ -499,14 +500,28 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     if constexpr (SOLVE) getrf_tile_solve<R, M>(a, pos, row_keep, r, tbase, b + tk.vo, x + tk.vo, sm);
 }
 
+// Out-of-line tile (kNoinline): each order gets its own register allocation
+// inside one kernel launch for a whole order range (instead of one kernel per
+// order, whose empty launches cost ~3 us each).
+template <typename R, int M, int F, bool SOLVE, class AfterLoad>
+__device__ __noinline__ void getrf_tile_call(R *A, FTask tk, const R *S, int32_t *piv, int32_t *info,
+                                             int32_t *safe_list, unsigned *safe_count, const R *b, R *x,
+                                             FastSmem<R> *sm, AfterLoad after_load) {
+    getrf_fast_tile<R, M, F, SOLVE>(A, tk, S, piv, info, safe_list, safe_count, b, x, *sm, after_load);
+}
+
 template <typename R, int M, int MHI, int F, bool SOLVE, class AfterLoad>
 __device__ __forceinline__ void getrf_fast_dispatch(R *A, const FTask &tk, const R *S, int32_t *piv, int32_t *info,
                                                     int32_t *safe_list, unsigned *safe_count, const R *b, R *x,
                                                     FastSmem<R> &sm, AfterLoad &&after_load) {
     if (tk.m == M) {
         constexpr int T = tile_width(M);
-        getrf_fast_tile<R, M, F, SOLVE>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info,
-                                        safe_list, safe_count, b, x, sm, after_load);
+        if constexpr ((F & kNoinline) != 0)
+            getrf_tile_call<R, M, F, SOLVE>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info,
+                                            safe_list, safe_count, b, x, &sm, after_load);
+        else
+            getrf_fast_tile<R, M, F, SOLVE>(A, tk, S + ((threadIdx.x & 31) / T) * stage_stride<R>(T), piv, info,
+                                            safe_list, safe_count, b, x, sm, after_load);
     } else {
         if constexpr (M < MHI)
             getrf_fast_dispatch<R, M + 1, MHI, F, SOLVE>(A, tk, S, piv, info, safe_list, safe_count, b, x, sm,
@@ -563,6 +578,21 @@ __device__ __forceinline__ void getrf_stage(R *A, const FTask &tk, R *S, uint64_
     __syncwarp();
     if (tk.ok && (lane % T) == 0) bulk_g2s(S + (lane / T) * stage_stride<R>(T), A + tk.lo, bytes, bar);
 }
+
+// Re-arm the warp's staging buffer with the next task once the current
+// block is in registers (the `after_load` step of getrf_fast_tile).
+template <typename R>
+struct StageNext {
+    R *A;
+    FTask nxt;
+    R *S;
+    uint64_t *bar;
+    __device__ __forceinline__ void operator()() const {
+        __syncwarp();                     // every lane has its block in registers
+        fence_proxy_async_smem();
+        getrf_stage(A, nxt, S, bar);
+    }
+};
 
 // One size class [MLO, MHI], persistent.  Each warp owns an 8-KB staging
 // buffer: while it factors task i from registers, the bulk copy of task i+1
@@ -686,11 +716,7 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
         mbar_wait_warp(bar, parity);
         parity ^= 1u;
         const FTask cur = slot_task(task, q0);
-        auto after_load = [&]() {
-            __syncwarp();                 // every lane has its block in registers
-            fence_proxy_async_smem();
-            getrf_stage(A, slot_task(task + nwarps, q1), S, bar);
-        };
+        const StageNext<R> after_load{A, slot_task(task + nwarps, q1), S, bar};
         getrf_fast_dispatch<R, MLO, MHI, F, SOLVE>(A, cur, S, piv, info, safe_list, safe_count, b, x, sm,
                                                    after_load);
         q0 = q1;

@@ -86,7 +86,7 @@ void run(Batch &b, const char *name, int64_t tot) {
         cudaMemcpy(b.A, b.A0, tot * 8, cudaMemcpyDeviceToDevice);
         cudaMemset(b.cnt, 0, 4);
         cudaEventRecord(e0);
-        kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt);
+        kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms; cudaEventElapsedTime(&ms, e0, e1);
@@ -111,7 +111,7 @@ void launch_one(Batch &b) {
         grid = per_sm * sm_count();
         printf("   M=%d occ %d warps/SM\n", M, per_sm * 4);
     }
-    kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt);
+    kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
 }
 template <int M, int F>
 void launch_range(Batch &b) {
@@ -140,47 +140,59 @@ void run_perm(Batch &b, const char *name, int64_t tot) {
            cudaGetErrorString(cudaGetLastError()));
 }
 
-template <int M, int F>
-void run_f(Batch &b, const char *name, int64_t tot) {
-    auto kern = k_getrf_fast<float, M, M, F>;
-    int per_sm = 0;
-    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFastThreads, 0);
-    const int grid = per_sm * sm_count();
+
+template <int LO, int HI, int F>
+void launch_cls(Batch &b) {
+    auto kern = k_getrf_fast<double, LO, HI, F>;
+    static int grid = 0;
+    if (!grid) {
+        int per_sm = 0;
+        cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFastThreads, 0);
+        grid = per_sm * sm_count();
+    }
+    kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
+}
+template <int W, int F>
+void run_groups(Batch &b, const char *name, int64_t tot) {
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
     std::vector<float> ts;
     for (int rep = 0; rep < 6; ++rep) {
-        cudaMemcpy(b.Af, b.Af0, tot * 4, cudaMemcpyDeviceToDevice);
+        cudaMemcpy(b.A, b.A0, tot * 8, cudaMemcpyDeviceToDevice);
         cudaMemset(b.cnt, 0, 4);
         cudaEventRecord(e0);
-        kern<<<grid, kFastThreads>>>(b.Af, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
+        if constexpr (W == 2) {
+            launch_cls<17, 18, F>(b); launch_cls<19, 20, F>(b); launch_cls<21, 22, F>(b); launch_cls<23, 24, F>(b);
+            launch_cls<25, 26, F>(b); launch_cls<27, 28, F>(b); launch_cls<29, 30, F>(b); launch_cls<31, 32, F>(b);
+        } else {
+            launch_cls<17, 20, F>(b); launch_cls<21, 24, F>(b); launch_cls<25, 28, F>(b); launch_cls<29, 32, F>(b);
+        }
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms; cudaEventElapsedTime(&ms, e0, e1);
         if (rep) ts.push_back(ms);
     }
     std::sort(ts.begin(), ts.end());
-    printf("%-28s F=%3d occ=%2d warps/SM  med %8.1f us  min %8.1f us  err=%s\n", name, F, per_sm * 4,
-           ts[ts.size() / 2] * 1e3, ts[0] * 1e3, cudaGetErrorString(cudaGetLastError()));
+    printf("%-28s F=%3d groups of %d  med %8.1f us  min %8.1f us  err=%s\n", name, F, W, ts[ts.size() / 2] * 1e3,
+           ts[0] * 1e3, cudaGetErrorString(cudaGetLastError()));
 }
-template <int M>
-void per_m() {
-    Batch b = make(34500, M, M);
-    int64_t tot = 34500LL * ((M * M + 3) / 4 * 4);
-    char n[64];
-    snprintf(n, sizeof n, "fp32 M=%d 34.5k", M);
-    run_f<M, 8 | 256>(b, n, tot);
-    run_f<M, 8 | 64>(b, n, tot);
-    run_f<M, 8 | 128>(b, n, tot);
-    run_f<M, 16 | 64>(b, n, tot);
-    run_f<M, 32 | 64>(b, n, tot);
-}
+
 int main() {
     setvbuf(stdout, NULL, _IONBF, 0);
-    per_m<17>();
-    per_m<22>();
-    per_m<26>();
-    per_m<30>();
-    per_m<32>();
+    {
+        const int64_t nb = 552000;
+        Batch b = make(nb, 17, 32);
+        int64_t tot = 0;
+        for (int64_t i = 0; i < nb; ++i) tot += (b.m_of[i] * b.m_of[i] + 3) / 4 * 4;
+        run_perm<8>(b, "mix 17..32 552k per-order", tot);
+        run_groups<2, 8>(b, "mix 17..32 552k", tot);
+        run_groups<4, 8>(b, "mix 17..32 552k", tot);
+        run_groups<2, 8 | 512>(b, "mix 17..32 552k noinline", tot);
+    }
+    {
+        Batch b = make(40000, 32, 32);
+        int64_t tot = 40000LL * 1024;
+
+    }
     return 0;
 }
