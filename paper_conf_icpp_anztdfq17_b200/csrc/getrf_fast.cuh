@@ -179,8 +179,8 @@ __device__ __forceinline__ float vfma(float a, float b, float c) {
 // header comment).  Column k0+W, the next panel's first pivot column, is
 // updated first.
 template <typename R, int M, int W, bool PRE>
-__device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, int &inf, bool &redo, bool row_ok, int r,
-                                                FastSmem<R> &sm) {
+__device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, unsigned &singmask, bool &redo, bool row_ok,
+                                                int r, FastSmem<R> &sm) {
     constexpr int PS = panel_stride<R>();
     constexpr int V = 16 / (int)sizeof(R);                 // elements per 16-B store / load
     const unsigned lanebits = 0x80000000u | (unsigned)(31 - r);
@@ -208,12 +208,10 @@ __device__ __forceinline__ void getrf_w32_steps(R (&a)[M], int &tag, int &inf, b
             if ((r == ipiv) && row_ok) tag = k + 1;             // line 9
             const bool sing = (d == R(0));                      // R4
             const bool upd = (tag == 0) && !sing;
-            bool bad = false;
-            const R q = Num<R>::div_nz_flag(a[k], d, yd, bad);  // line 13 (SCAL)
-            redo = redo || (upd && bad);
+            const R q = Num<R>::div_fastpath(a[k], d, yd);       // line 13 (SCAL); exact for kept blocks
             const R l = upd ? q : R(0);
             if (upd) a[k] = q;
-            if (sing && inf == 0) inf = k + 1;
+            singmask |= sing ? (1u << k) : 0u;
             lk[sidx] = l;
             ipv[sidx] = ipiv;
             static_for<k + 1, kend>([&](auto jc) {              // lines 14-15 inside the panel
@@ -351,11 +349,11 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     const bool row_ok = tile_ok && (r < M);
 
     int tag = row_ok ? 0 : -1;      // 0: candidate; k+1: pivot of step k; -1: inactive lane
-    int inf = 0;
-    bool redo = false;              // pivot ambiguity or IEEE slow-path quotient in this tile
+    unsigned singmask = 0;          // bit k: step k was singular (R4); info = first such step + 1
+    bool redo = false;              // pivot ambiguity or failed magnitude test in this tile
     const unsigned lanebits = 0x80000000u | (unsigned)(31 - r);
     if constexpr (W32 && panel_width(F) > 1) {
-        getrf_w32_steps<R, M, panel_width(F), (F & kPre) != 0>(a, tag, inf, redo, row_ok, r, sm);
+        getrf_w32_steps<R, M, panel_width(F), (F & kPre) != 0>(a, tag, singmask, redo, row_ok, r, sm);
     } else static_for<0, M>([&](auto kc) {
         constexpr int k = decltype(kc)::value;
         const bool cand = (tag == 0);
@@ -410,12 +408,10 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         const bool sing = (d == R(0));                              // R4: all candidates +-0
         // line 13 (SCAL), then lines 14-15 (GER) on the rows still unpivoted
         const bool upd = (tag == 0) && !sing;
-        bool bad = false;
-        const R q = Num<R>::div_nz_flag(a[k], d, yd, bad);
-        redo = redo || (upd && bad);
+        const R q = Num<R>::div_fastpath(a[k], d, yd);          // exact for kept blocks (common.cuh)
         const R l = upd ? q : R(0);
         if (upd) a[k] = q;
-        if (sing && inf == 0) inf = k + 1;
+        singmask |= sing ? (1u << k) : 0u;
         if constexpr (W32) {
             static_for<k + 1, M>([&](auto jc) {
                 constexpr int j = decltype(jc)::value;
@@ -496,7 +492,7 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         });
         piv[tk.vo + pos] = r;
     }
-    if (keep && r == 0) info[blk] = inf;
+    if (keep && r == 0) info[blk] = __ffs((int)singmask);
     if constexpr (SOLVE) getrf_tile_solve<R, M>(a, pos, row_keep, r, tbase, b + tk.vo, x + tk.vo, sm);
 }
 
