@@ -78,6 +78,12 @@ def _declare(L):
         getattr(L, f"bjo_getri_batch_{s}").restype = None
         getattr(L, f"bjo_gemv_batch_{s}").argtypes = [_i64, _p, _p, _p, _p, _p, _p, _i32]
         getattr(L, f"bjo_gemv_batch_{s}").restype = None
+    L.bjo_spmv_d.argtypes = [_i64, _p, _p, _p, _i64, _p, _p]
+    L.bjo_spmv_d.restype = None
+    L.bjo_dot_d.argtypes = [_i64, _p, _p]
+    L.bjo_dot_d.restype = ctypes.c_double
+    L.bjo_bicgstab_d.argtypes = [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_double, _i32, _p, _p]
+    L.bjo_bicgstab_d.restype = _i32
     L.bjo_layout.argtypes = [_i64, _p, _i32, _p, _p]
     L.bjo_layout.restype = None
     L.bjo_extract.argtypes = [_i64, _p, _p, _p, _i32, _i64, _i64, _p, _p, _p]
@@ -235,6 +241,44 @@ def gemv_batch(sizes, val_off, vec_off, Dinv, x, nthreads: int = 0):
     getattr(lib(), f"bjo_gemv_batch_{s}")(nb, _ptr(sizes), _ptr(val_off), _ptr(vec_off),
                                           _ptr(Dinv), _ptr(x), _ptr(y), int(nthreads))
     return y[: int(vec_off[nb])]
+
+
+def spmv(row_ptr, col_idx, values, x, col_offset: int = 0):
+    """y = A x with the fixed summation order R27 (fp64)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    values = np.ascontiguousarray(values, dtype=np.float64)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    n = row_ptr.shape[0] - 1
+    y = np.zeros(max(n, 1))
+    lib().bjo_spmv_d(n, _ptr(row_ptr), _ptr(col_idx), _ptr(values), int(col_offset), _ptr(x), _ptr(y))
+    return y[:n]
+
+
+def dot(x, y) -> float:
+    """dot product with the fixed chunked order R28 (fp64)."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.ascontiguousarray(y, dtype=np.float64)
+    return float(lib().bjo_dot_d(x.shape[0], _ptr(x), _ptr(y)))
+
+
+def bicgstab(row_ptr, col_idx, values, block_ptr, b, tol: float = 1e-6, maxit: int = 10000,
+             col_offset: int = 0):
+    """Block-Jacobi (LU) preconditioned BiCGSTAB, R27-R29 (section IV.D,
+    P:852-856).  Returns (x, iterations, relative residual, LU, perm, info)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    values = np.ascontiguousarray(values, dtype=np.float64)
+    D, sizes, vec, val = extract(row_ptr, col_idx, values, block_ptr, col_offset)
+    LU, perm, info = getrf_batch(sizes, val, vec, D)
+    n = row_ptr.shape[0] - 1
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    x = np.zeros(max(n, 1))
+    res = ctypes.c_double(0.0)
+    it = lib().bjo_bicgstab_d(n, _ptr(row_ptr), _ptr(col_idx), _ptr(values), int(col_offset), len(sizes),
+                              _ptr(sizes), _ptr(val), _ptr(vec), _ptr(LU), _ptr(perm), _ptr(b), float(tol),
+                              int(maxit), _ptr(x), ctypes.byref(res))
+    return x[:n], int(it), float(res.value), LU, perm, info
 
 
 def extract(row_ptr, col_idx, values, block_ptr, col_offset: int = 0):
