@@ -84,6 +84,11 @@ def _declare(L):
     L.bjo_dot_d.restype = ctypes.c_double
     L.bjo_bicgstab_d.argtypes = [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_double, _i32, _p, _p]
     L.bjo_bicgstab_d.restype = _i32
+    L.bjo_dot_sharded_d.argtypes = [_i64, _p, _p, _i32, _p]
+    L.bjo_dot_sharded_d.restype = ctypes.c_double
+    L.bjo_bicgstab_sharded_d.argtypes = [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_double,
+                                         _i32, _i32, _p, _p, _p]
+    L.bjo_bicgstab_sharded_d.restype = _i32
     L.bjo_layout.argtypes = [_i64, _p, _i32, _p, _p]
     L.bjo_layout.restype = None
     L.bjo_extract.argtypes = [_i64, _p, _p, _p, _i32, _i64, _i64, _p, _p, _p]
@@ -262,10 +267,19 @@ def dot(x, y) -> float:
     return float(lib().bjo_dot_d(x.shape[0], _ptr(x), _ptr(y)))
 
 
+def dot_sharded(x, y, bounds) -> float:
+    """R30: per-shard R28 dots summed in shard order from +0."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.ascontiguousarray(y, dtype=np.float64)
+    b = np.ascontiguousarray(bounds, dtype=np.int64)
+    return float(lib().bjo_dot_sharded_d(x.shape[0], _ptr(x), _ptr(y), b.shape[0] - 1, _ptr(b)))
+
+
 def bicgstab(row_ptr, col_idx, values, block_ptr, b, tol: float = 1e-6, maxit: int = 10000,
-             col_offset: int = 0):
+             col_offset: int = 0, bounds=None):
     """Block-Jacobi (LU) preconditioned BiCGSTAB, R27-R29 (section IV.D,
-    P:852-856).  Returns (x, iterations, relative residual, LU, perm, info)."""
+    P:852-856); with `bounds` (row shards, int64[G+1]) the dots follow R30.
+    Returns (x, iterations, relative residual, LU, perm, info)."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     values = np.ascontiguousarray(values, dtype=np.float64)
@@ -275,9 +289,16 @@ def bicgstab(row_ptr, col_idx, values, block_ptr, b, tol: float = 1e-6, maxit: i
     b = np.ascontiguousarray(b, dtype=np.float64)
     x = np.zeros(max(n, 1))
     res = ctypes.c_double(0.0)
-    it = lib().bjo_bicgstab_d(n, _ptr(row_ptr), _ptr(col_idx), _ptr(values), int(col_offset), len(sizes),
-                              _ptr(sizes), _ptr(val), _ptr(vec), _ptr(LU), _ptr(perm), _ptr(b), float(tol),
-                              int(maxit), _ptr(x), ctypes.byref(res))
+    if bounds is None:
+        it = lib().bjo_bicgstab_d(n, _ptr(row_ptr), _ptr(col_idx), _ptr(values), int(col_offset), len(sizes),
+                                  _ptr(sizes), _ptr(val), _ptr(vec), _ptr(LU), _ptr(perm), _ptr(b), float(tol),
+                                  int(maxit), _ptr(x), ctypes.byref(res))
+    else:
+        bd = np.ascontiguousarray(bounds, dtype=np.int64)
+        it = lib().bjo_bicgstab_sharded_d(n, _ptr(row_ptr), _ptr(col_idx), _ptr(values), int(col_offset),
+                                          len(sizes), _ptr(sizes), _ptr(val), _ptr(vec), _ptr(LU), _ptr(perm),
+                                          _ptr(b), float(tol), int(maxit), bd.shape[0] - 1, _ptr(bd), _ptr(x),
+                                          ctypes.byref(res))
     return x[:n], int(it), float(res.value), LU, perm, info
 
 

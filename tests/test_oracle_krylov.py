@@ -84,3 +84,39 @@ def test_bicgstab_fem_block_jacobi():
     # not converged within maxit -> maxit + 1
     _, it2, res2, *_ = oracle.bicgstab(rp, ci, va, bp, b, tol=1e-30, maxit=3)
     assert it2 == 4 and res2 > 1e-30
+
+
+def test_dot_sharded_r30():
+    """R30: per-shard R28 values summed in shard order from +0; one shard is R28."""
+    rng = np.random.default_rng(54)
+    z = rng.uniform(-1, 1, 30000)
+    w = rng.uniform(-1, 1, 30000)
+    assert oracle.dot_sharded(z, w, [0, 30000]) == oracle.dot(z, w)
+    bnd = [0, 7001, 7001, 19999, 30000]                      # an empty shard too
+    manual = 0.0
+    for a, b in zip(bnd[:-1], bnd[1:]):
+        manual = manual + oracle.dot(z[a:b], w[a:b])
+    assert oracle.dot_sharded(z, w, bnd) == manual
+    zi = rng.integers(-50, 51, 30000).astype(np.float64)
+    assert oracle.dot_sharded(zi, zi, bnd) == float(np.dot(zi.astype(np.int64), zi.astype(np.int64)))
+    # order pin: elements (1, 2^-53, 0, 2^-53).  One chunk: the tree adds positions
+    # 1 and 3 first (2^-52), then 1 + 2^-52.  Shards [0,1) [1,2) [2,4): 1 + 2^-53 + 2^-53 -> 1.
+    x = np.array([1.0, 2.0 ** -53, 0.0, 2.0 ** -53])
+    assert oracle.dot(x, np.ones(4)) == 1.0 + 2.0 ** -52
+    assert oracle.dot_sharded(x, np.ones(4), [0, 1, 2, 4]) == 1.0
+
+
+def test_bicgstab_sharded_r30():
+    g = S.FemGrid(10, 9, 8)
+    rp, ci, va = g.csr()
+    n = g.n
+    bp = S.uniform_block_ptr(n, 24)
+    b = np.ones(n)
+    x1, it1, res1, *_ = oracle.bicgstab(rp, ci, va, bp, b)
+    xs, its, ress, *_ = oracle.bicgstab(rp, ci, va, bp, b, bounds=[0, n])
+    assert its == it1 and ress == res1 and np.array_equal(xs.view(np.uint64), x1.view(np.uint64))
+    bnd = [0, 3 * 10 * 9 * 3, 3 * 10 * 9 * 5, n]            # z-slab shards
+    x3, it3, res3, *_ = oracle.bicgstab(rp, ci, va, bp, b, bounds=bnd)
+    A = sp.csr_matrix((va, ci, rp), shape=(n, n))
+    assert res3 <= 1e-6 and np.linalg.norm(b - A @ x3) / np.linalg.norm(b) <= 2e-6
+    assert abs(it3 - it1) <= 2
