@@ -51,7 +51,8 @@ typedef enum {
     BJ_ERR_ALIGN = -3,       /* a base pointer is not 16-byte aligned          */
     BJ_ERR_CUDA = -4,        /* a CUDA runtime call or launch failed           */
     BJ_ERR_NOMEM = -5,       /* library scratch allocation failed              */
-    BJ_ERR_STATE = -6        /* handle used before bj_setup, ...               */
+    BJ_ERR_STATE = -6,       /* handle used before bj_setup, ...               */
+    BJ_ERR_COMM = -7         /* a bj_comm callback reported failure             */
 } bj_status;
 
 /* Sparse matrix in CSR (CSR [3]; Fig. 3).  Rows are
@@ -260,6 +261,86 @@ bj_status bj_supervariable_blocking(const bj_csr *A, int32_t max_block, int32_t 
  * ------------------------------------------------------------------------- */
 bj_status bj_selftest_div(bj_dtype dtype, int64_t n, uint64_t seed, uint64_t *counts_h, void *sample_h,
                           int64_t nsample);
+
+/* ---------------------------------------------------------------------------
+ * NEXT(4) -- block-Jacobi preconditioned Krylov solve, the paper's end-to-end
+ * use of the preconditioner (section IV.D: right-hand side of all
+ * ones, initial guess zero, stop once the relative residual norm has dropped
+ * by six orders of magnitude, at most 10,000 iterations; the
+ * preconditioner is applied "once per step of the iterative solve").  The
+ * paper runs IDR(4); this build runs BiCGSTAB (reading R29).  fp64 only
+ * (A->dtype must be BJ_F64).  Every reduction has a fixed order, so results
+ * are reproducible bit for bit and equal to the oracle's:
+ *
+ * bj_spmv:  y = A x (R27).  Row i: lane l of a warp accumulates
+ *   s_l = fma(val_e, x[col_e - col_offset], s_l) over the row's entries
+ *   e = row_ptr[i] + l, + l + 32, ... in order, from +0; then
+ *   s_l += s_(l^16), s_l += s_(l^8), ..., s_l += s_(l^1); y_i = s_0.
+ *   x has at least max(col_idx) - col_offset + 1 elements; y (A->nrows) must
+ *   not overlap x.
+ * bj_dot:  *result (a DEVICE double) = dot(x, y) over n elements (R28): chunks
+ *   of 8192 consecutive elements; thread t of 256 accumulates
+ *   fma(x_k, y_k, s_t) over k = chunk + t + 256 j (j = 0..31) from +0; the
+ *   256 partials are added by the tree s_t += s_(t+h), h = 128, ..., 1; the
+ *   chunk sums are added in chunk order from +0.
+ * bj_bicgstab: solves A x = b with right-preconditioned BiCGSTAB, M^-1 =
+ *   bj_apply(M, .) (a handle set up by bj_setup or bj_setup_inverse on the
+ *   same rows; the oracle pins the LU handle).  r = rh = b, p = v = 0, x = 0,
+ *   rho_prev = alpha = omega = 1; per iteration
+ *     rho = dot(rh, r); beta = (rho / rho_prev) * (alpha / omega);
+ *     p = fma(beta, fma(-omega, v, p), r); ph = M^-1 p; v = A ph;
+ *     alpha = rho / dot(rh, v); s = fma(-alpha, v, r); sh = M^-1 s; t = A sh;
+ *     omega = dot(t, s) / dot(t, t); x = fma(omega, sh, fma(alpha, ph, x));
+ *     r = fma(-omega, t, s); stop if sqrt(dot(r, r)) <= tol * sqrt(dot(b, b));
+ *     rho_prev = rho.
+ *   The loop runs on the device (scalars in device memory, no host round
+ *   trip per iteration; the host polls a completion flag two iterations
+ *   behind).  *iters_h (HOST) = the iteration that converged, or maxit + 1;
+ *   *resid_h (HOST) = final ||r|| / ||b||.  x (A->nrows) is overwritten; b
+ *   is read only.  Synchronous on return.  Scratch: 9 vectors of A->nrows
+ *   (+ halo) doubles (cudaMallocAsync).
+ *   comm = NULL: one GPU, A holds every column (col_offset as in bj_csr).
+ *   comm != NULL (rows sharded over comm->nranks processes): A's col_idx are
+ *   LOCAL EXTENDED ids from bj_halo_plan (own rows 0..nrows-1, then the halo)
+ *   and A->col_offset must be 0.  Before each SpMV the library packs
+ *   x[send_idx[j]] into comm->send_buf and calls halo_exchange(ctx, stream),
+ *   which must deliver every peer's entries into comm->recv_buf in halo order
+ *   (stream-ordered).  For each dot the library writes its k <= 4 rank sums
+ *   to gather_buf[rank*4 .. rank*4+k) and calls allgather(ctx, k, stream),
+ *   which must fill every rank's row; the global value is the sum over ranks
+ *   in rank order from +0 (reading R30; one rank reproduces R28 exactly).
+ *   A callback returning nonzero aborts with BJ_ERR_COMM.
+ * bj_halo_plan (HOST): for rows [lo, hi) of a matrix whose rows are sharded
+ *   as row_bounds_h[0..G] (rank q owns [row_bounds_h[q], row_bounds_h[q+1])),
+ *   maps the nnz global column ids col_idx_h to col_local_h: c - lo for an
+ *   own column, (hi - lo) + j for the j-th distinct remote column in
+ *   ascending order.  halo_cols_h (capacity nnz) receives those distinct
+ *   remote columns in ascending order, *nhalo_h their count and
+ *   recv_counts_h[q] (G entries) how many of them rank q owns (so the halo is
+ *   grouped by owner, in rank order).  A column outside [0, row_bounds_h[G])
+ *   is BJ_ERR_ARG.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    void *ctx;
+    int nranks;
+    int rank;
+    int64_t nhalo;              /* halo entries received (x extension length)   */
+    int64_t nsend;              /* entries sent to peers                        */
+    const int32_t *send_idx;    /* device [nsend]: own rows to send, by peer     */
+    double *send_buf;           /* device [nsend], caller-owned                 */
+    double *recv_buf;           /* device [nhalo], caller-owned                 */
+    double *gather_buf;         /* device [nranks * 4], caller-owned            */
+    int (*halo_exchange)(void *ctx, bj_stream_t stream);
+    int (*allgather)(void *ctx, int k, bj_stream_t stream);
+} bj_comm;
+
+bj_status bj_spmv(const bj_csr *A, const double *x, double *y, bj_stream_t stream);
+bj_status bj_dot(int64_t n, const double *x, const double *y, double *result, bj_stream_t stream);
+bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *comm, const double *b, double *x,
+                      double tol, int maxit, int *iters_h, double *resid_h, bj_stream_t stream);
+bj_status bj_halo_plan(int64_t nnz, const int32_t *col_idx_h, int64_t lo, int64_t hi, int G,
+                       const int64_t *row_bounds_h, int32_t *col_local_h, int32_t *halo_cols_h,
+                       int64_t *nhalo_h, int64_t *recv_counts_h);
 
 /* ---------------------------------------------------------------------------
  * End-to-end call with HOST buffers (synchronous): copies sizes_h (nblocks),

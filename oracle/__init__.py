@@ -84,6 +84,8 @@ def _declare(L):
     L.bjo_dot_d.restype = ctypes.c_double
     L.bjo_bicgstab_d.argtypes = [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_double, _i32, _p, _p]
     L.bjo_bicgstab_d.restype = _i32
+    L.bjo_fma_vec.argtypes = [_i64, _p, _p, _p, _p]
+    L.bjo_fma_vec.restype = None
     L.bjo_dot_sharded_d.argtypes = [_i64, _p, _p, _i32, _p]
     L.bjo_dot_sharded_d.restype = ctypes.c_double
     L.bjo_bicgstab_sharded_d.argtypes = [_i64, _p, _p, _p, _i64, _i64, _p, _p, _p, _p, _p, _p, ctypes.c_double,
@@ -265,6 +267,16 @@ def dot(x, y) -> float:
     x = np.ascontiguousarray(x, dtype=np.float64)
     y = np.ascontiguousarray(y, dtype=np.float64)
     return float(lib().bjo_dot_d(x.shape[0], _ptr(x), _ptr(y)))
+
+
+def fma_vec(a, x, y):
+    """out = fma(a, x, y) elementwise (C99 fma, single rounding)."""
+    a = np.ascontiguousarray(a, dtype=np.float64)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.ascontiguousarray(y, dtype=np.float64)
+    out = np.empty(max(x.shape[0], 1))
+    lib().bjo_fma_vec(x.shape[0], _ptr(a), _ptr(x), _ptr(y), _ptr(out))
+    return out[: x.shape[0]]
 
 
 def dot_sharded(x, y, bounds) -> float:

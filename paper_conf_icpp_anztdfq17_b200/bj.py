@@ -19,7 +19,7 @@ LIB_PATH = os.path.join(_HERE, "libbj.so")
 
 BJ_F32, BJ_F64 = 0, 1
 _STATUS = {0: "BJ_OK", -1: "BJ_ERR_ARG", -2: "BJ_ERR_BLOCK_SIZE", -3: "BJ_ERR_ALIGN", -4: "BJ_ERR_CUDA",
-           -5: "BJ_ERR_NOMEM", -6: "BJ_ERR_STATE"}
+           -5: "BJ_ERR_NOMEM", -6: "BJ_ERR_STATE", -7: "BJ_ERR_COMM"}
 
 # every symbol include/bj.h and include/bj_synth.h declare
 EXPORTS = (
@@ -29,6 +29,7 @@ EXPORTS = (
     "bj_create", "bj_setup",
     "bj_apply", "bj_destroy", "bj_partition", "bj_workspace_create", "bj_workspace_destroy", "bj_gesv_host",
     "bj_launch_count", "bj_launch_count_reset", "bj_supervariable_blocking",
+    "bj_spmv", "bj_dot", "bj_bicgstab", "bj_halo_plan",
     "bj_synth_sizes", "bj_synth_blocks", "bj_synth_rhs", "bj_synth_fem_row_ptr", "bj_synth_fem_fill",
 )
 
@@ -41,6 +42,17 @@ class CSR(ctypes.Structure):
     _fields_ = [("nrows", ctypes.c_int64), ("nnz", ctypes.c_int64), ("col_offset", ctypes.c_int64),
                 ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("values", ctypes.c_void_p),
                 ("dtype", ctypes.c_int)]
+
+
+HALO_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+GATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_int, ctypes.c_void_p)
+
+
+class CommC(ctypes.Structure):
+    _fields_ = [("ctx", ctypes.c_void_p), ("nranks", ctypes.c_int), ("rank", ctypes.c_int),
+                ("nhalo", ctypes.c_int64), ("nsend", ctypes.c_int64), ("send_idx", ctypes.c_void_p),
+                ("send_buf", ctypes.c_void_p), ("recv_buf", ctypes.c_void_p), ("gather_buf", ctypes.c_void_p),
+                ("halo_exchange", HALO_FN), ("allgather", GATHER_FN)]
 
 
 class BatchC(ctypes.Structure):
@@ -84,6 +96,10 @@ def lib() -> ctypes.CDLL:
             "bj_workspace_create": ([P], I32),
             "bj_workspace_destroy": ([P], I32),
             "bj_gesv_host": ([P, I64, P, I64, P, I64, P, P, P, P, I32, P], I32),
+            "bj_spmv": ([P, P, P, P], I32),
+            "bj_dot": ([I64, P, P, P, P], I32),
+            "bj_bicgstab": ([P, P, P, P, P, ctypes.c_double, I32, P, P, P], I32),
+            "bj_halo_plan": ([I64, P, I64, I64, I32, P, P, P, P, P], I32),
             "bj_launch_count": ([], I64),
             "bj_launch_count_reset": ([], None),
             "bj_synth_sizes": ([I64, I64, I32, I32, ctypes.c_uint64, P, P], I32),
@@ -399,3 +415,131 @@ def selftest_div(dtype: torch.dtype, n: int, seed: int = 1, nsample: int = 0):
     _check(lib().bj_selftest_div(dtype_code(dtype), int(n), int(seed), counts.ctypes.data_as(ctypes.c_void_p),
                                  sample.ctypes.data_as(ctypes.c_void_p), int(nsample)), "bj_selftest_div")
     return counts, sample[:nsample]
+
+
+# ---------------------------------------------------------------------------
+# NEXT(4): block-Jacobi preconditioned BiCGSTAB (section IV.D, R27-R30)
+
+def spmv(A: Csr, x: torch.Tensor, y: torch.Tensor, stream=None):
+    """y = A x in the fixed order R27 (fp64)."""
+    a = A.c()
+    _check(lib().bj_spmv(ctypes.byref(a), _p(x), _p(y), _stream(stream)), "bj_spmv")
+
+
+def dot(x: torch.Tensor, y: torch.Tensor, stream=None) -> torch.Tensor:
+    """dot(x, y) in the fixed order R28 (fp64); returns a 0-d device tensor."""
+    out = torch.empty((), dtype=torch.float64, device=x.device)
+    _check(lib().bj_dot(x.numel(), _p(x), _p(y), _p(out), _stream(stream)), "bj_dot")
+    return out
+
+
+def halo_plan(col_idx_h: np.ndarray, lo: int, hi: int, row_bounds: np.ndarray):
+    """Host halo plan (bj_halo_plan): (col_local int32[nnz], halo_cols
+    int32[nhalo] ascending, recv_counts int64[G])."""
+    ci = np.ascontiguousarray(col_idx_h, dtype=np.int32)
+    rb = np.ascontiguousarray(row_bounds, dtype=np.int64)
+    G = rb.shape[0] - 1
+    cl = np.empty(max(ci.shape[0], 1), dtype=np.int32)
+    hc = np.empty(max(ci.shape[0], 1), dtype=np.int32)
+    nh = ctypes.c_int64(0)
+    rc = np.zeros(G, dtype=np.int64)
+    vp = ctypes.c_void_p
+    _check(lib().bj_halo_plan(ci.shape[0], ci.ctypes.data_as(vp), int(lo), int(hi), G, rb.ctypes.data_as(vp),
+                              cl.ctypes.data_as(vp), hc.ctypes.data_as(vp), ctypes.byref(nh),
+                              rc.ctypes.data_as(vp)), "bj_halo_plan")
+    return cl[: ci.shape[0]], hc[: nh.value].copy(), rc
+
+
+class TorchComm:
+    """bj_comm over torch.distributed (NCCL on GPUs, gloo on CPU): the halo
+    exchange is one all_to_all_single, the dot combination one
+    all_gather_into_tensor.  Built once from this rank's halo plan: the
+    requested column ids are exchanged so every rank knows what to send."""
+
+    def __init__(self, halo_cols: np.ndarray, recv_counts: np.ndarray, lo: int, device, group=None):
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.rank, self.nranks = dist.get_rank(group), dist.get_world_size(group)
+        self.device = torch.device(device)
+        rc = torch.as_tensor(np.asarray(recv_counts, dtype=np.int64), device=self.device)
+        sc = torch.empty_like(rc)
+        dist.all_to_all_single(sc, rc, group=group)                   # how many each peer wants from me
+        self.recv_counts = [int(v) for v in rc.tolist()]
+        self.send_counts = [int(v) for v in sc.tolist()]
+        req = torch.as_tensor(np.asarray(halo_cols, dtype=np.int32), device=self.device)
+        want = torch.empty(sum(self.send_counts), dtype=torch.int32, device=self.device)
+        dist.all_to_all_single(want, req, output_split_sizes=self.send_counts,
+                               input_split_sizes=self.recv_counts, group=group)
+        self.send_idx = (want.long() - int(lo)).to(torch.int32)       # own rows to send, by peer
+        self.send_buf = torch.zeros(max(want.numel(), 1), dtype=torch.float64, device=self.device)
+        self.recv_buf = torch.zeros(max(req.numel(), 1), dtype=torch.float64, device=self.device)
+        self.gather_buf = torch.zeros(self.nranks * 4, dtype=torch.float64, device=self.device)
+        self.nsend, self.nhalo = want.numel(), req.numel()
+        self._halo_cb = HALO_FN(self._halo)
+        self._gather_cb = GATHER_FN(self._gather)
+
+    def halo_exchange(self):
+        """send_buf -> recv_buf (grouped by owner rank, halo order)."""
+        self.dist.all_to_all_single(self.recv_buf[: self.nhalo], self.send_buf[: self.nsend],
+                                    output_split_sizes=self.recv_counts, input_split_sizes=self.send_counts,
+                                    group=self.group)
+
+    def allgather(self, k: int):
+        """every rank's row gather_buf[r*4 : r*4+4] to every rank."""
+        mine = self.gather_buf[self.rank * 4: self.rank * 4 + 4].clone()
+        self.dist.all_gather_into_tensor(self.gather_buf, mine, group=self.group)
+
+    def _halo(self, ctx, stream):
+        try:
+            self.halo_exchange()
+            return 0
+        except Exception:
+            return 1
+
+    def _gather(self, ctx, k, stream):
+        try:
+            self.allgather(int(k))
+            return 0
+        except Exception:
+            return 1
+
+    def c(self) -> CommC:
+        return CommC(None, self.nranks, self.rank, self.nhalo, self.nsend, _p(self.send_idx), _p(self.send_buf),
+                     _p(self.recv_buf), _p(self.gather_buf), self._halo_cb, self._gather_cb)
+
+
+class LoopbackComm(TorchComm):
+    """One-rank bj_comm without torch.distributed (exercises the library's
+    communication path on a single GPU: empty halo, identity allgather)."""
+
+    def __init__(self, device="cuda"):
+        self.rank, self.nranks, self.device = 0, 1, torch.device(device)
+        self.send_idx = torch.zeros(1, dtype=torch.int32, device=self.device)
+        self.send_buf = torch.zeros(1, dtype=torch.float64, device=self.device)
+        self.recv_buf = torch.zeros(1, dtype=torch.float64, device=self.device)
+        self.gather_buf = torch.zeros(4, dtype=torch.float64, device=self.device)
+        self.nsend = self.nhalo = 0
+        self.calls = {"halo": 0, "allgather": 0}
+        self._halo_cb = HALO_FN(self._halo)
+        self._gather_cb = GATHER_FN(self._gather)
+
+    def halo_exchange(self):
+        self.calls["halo"] += 1
+
+    def allgather(self, k: int):
+        self.calls["allgather"] += 1
+
+
+def bicgstab(M: Handle, A: Csr, b: torch.Tensor, x: torch.Tensor, tol: float = 1e-6, maxit: int = 10000,
+             comm: TorchComm | None = None, stream=None):
+    """NEXT(4): block-Jacobi (M = a set-up Handle) preconditioned BiCGSTAB,
+    R29 / R30.  x is overwritten.  Returns (iterations, relative residual);
+    iterations = maxit + 1 when not converged.  Synchronous."""
+    a = A.c()
+    it = ctypes.c_int(0)
+    res = ctypes.c_double(0.0)
+    cc = comm.c() if comm is not None else None
+    _check(lib().bj_bicgstab(M._h, ctypes.byref(a), ctypes.byref(cc) if cc is not None else None, _p(b), _p(x),
+                             float(tol), int(maxit), ctypes.byref(it), ctypes.byref(res), _stream(stream)),
+           "bj_bicgstab")
+    return it.value, res.value

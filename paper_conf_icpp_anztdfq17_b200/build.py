@@ -32,7 +32,7 @@ DTYPES = ["double", "float"]
 
 def _jobs():
     jobs = []
-    for src in ("api.cu", "layout.cu", "getrf.cu", "getrs.cu", "extract.cu", "synth.cu", "supervar.cu", "getri.cu", "selftest.cu"):
+    for src in ("api.cu", "layout.cu", "getrf.cu", "getrs.cu", "extract.cu", "synth.cu", "supervar.cu", "getri.cu", "selftest.cu", "krylov.cu"):
         jobs.append((src, [], src.replace(".cu", ".o")))
     for kind in ("getrf", "getrs"):
         for dt in DTYPES:

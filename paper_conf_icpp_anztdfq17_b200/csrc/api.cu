@@ -105,6 +105,7 @@ const char *bj_status_string(bj_status st) {
     case BJ_ERR_CUDA: return "BJ_ERR_CUDA: CUDA runtime error";
     case BJ_ERR_NOMEM: return "BJ_ERR_NOMEM: allocation failed";
     case BJ_ERR_STATE: return "BJ_ERR_STATE: object not ready";
+    case BJ_ERR_COMM: return "BJ_ERR_COMM: communication callback failed";
     }
     return "unknown bj_status";
 }
