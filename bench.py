@@ -33,7 +33,7 @@ import torch.distributed as dist
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22), "SV": (174, 174, 22)}   # per-GPU z-slab of 22 planes
+FEM = {"C4": (174, 174, 22), "C5": (174, 174, 22), "SV": (174, 174, 22), "C5K": (174, 174, 22)}   # per-GPU z-slab of 22 planes
 
 CONFIGS = {
     # name: (nblocks per GPU, lo, hi, dtype, description)
@@ -43,6 +43,8 @@ CONFIGS = {
     "C1": (1_000, 4, 16, torch.float64, "C1: 1,000 blocks m ~ U{4..16}, fp64 (latency case, L2-resident)"),
     "C4": (0, 24, 24, torch.float64, "C4: diagonal-block extraction, 27-pt x 3-dof FEM CSR, 1,998,216 rows/GPU, skewed hubs"),
     "C5": (0, 24, 24, torch.float64, "C5: block-Jacobi setup (extract + getrf) + 100 applies, 1,998,216 rows/GPU, b = 24"),
+    "C5K": (0, 24, 24, torch.float64, "C5K (NEXT 4): block-Jacobi setup + BiCGSTAB solve (b = ones, x0 = 0, 1e-6 reduction) "
+                                      "on the 27-pt x 3-dof FEM matrix, 1,998,216 rows/GPU (z-slabs, halo exchange), b = 24"),
     "SV": (0, 24, 24, torch.float64, "SV (NEXT 2): supervariable blocking of the C4 CSR pattern, 1,998,216 rows/GPU, bound 24"),
 }
 
@@ -602,6 +604,121 @@ def run_fem(args, ws, rank, local):
         print(json.dumps(line), flush=True)
 
 
+def run_krylov(args, ws, rank, local):
+    """C5K (NEXT 4): block-Jacobi setup + preconditioned BiCGSTAB solve of
+    the section IV.D set-up on a 174 x 174 x (22 * ws) FEM grid,
+    rank r owning the r-th 22-plane z-slab (weak scaling; halo exchange and
+    rank-ordered dot sums through bj.TorchComm over NCCL when ws > 1)."""
+    from paper_conf_icpp_anztdfq17_b200 import bj
+    nx, ny, nzr = FEM["C5K"]
+    b = args.block or 24
+    dt = torch.float64
+    nz = nzr * ws
+    plane = 3 * nx * ny
+    r0, r1 = rank * nzr * plane, (rank + 1) * nzr * plane
+    n = r1 - r0
+    A = bj.synth_fem(nx, ny, nz, r0, r1, dtype=dt)            # local rows, global columns
+    nnz = A.col_idx.numel()
+    bp = torch.arange(0, n + b, b, dtype=torch.int32, device="cuda").clamp_(max=n)
+    bp = torch.unique_consecutive(bp)
+    nb = bp.numel() - 1
+    sizes, vec, val = bj.layout_from_block_ptr(bp, dt)
+    fac = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=dt, device="cuda"))
+    piv = torch.empty(n, dtype=torch.int32, device="cuda")
+    info = torch.empty(nb, dtype=torch.int32, device="cuda")
+    comm = None
+    Aloc = bj.Csr(A.row_ptr, A.col_idx, A.values, 0)           # SpMV view: column ids as stored
+    if ws > 1:
+        bounds = np.arange(ws + 1, dtype=np.int64) * n
+        cl, hc, rc = bj.halo_plan(A.col_idx.cpu().numpy(), r0, r1, bounds)
+        comm = bj.TorchComm(hc, rc, r0, "cuda")
+        Aloc = bj.Csr(A.row_ptr, torch.from_numpy(cl).cuda(), A.values, 0)
+    rhs = torch.ones(n, dtype=dt, device="cuda")
+    x = torch.empty(n + (comm.nhalo if comm else 0), dtype=dt, device="cuda")
+    xs = torch.rand(n + (comm.nhalo if comm else 0), dtype=dt, device="cuda") * 2 - 1
+    ys = torch.empty(n, dtype=dt, device="cuda")
+    h = bj.Handle()
+    stream = torch.cuda.current_stream()
+    hbm, peak_src = load_peaks()
+    iters = [0]
+
+    def step(evs=None):
+        if evs is not None:
+            evs[0].record(stream)
+        h.setup(A, bp, fac, piv, info)                         # extract + GETRF (fused for m = 17..32)
+        if evs is not None:
+            evs[1].record(stream)
+        it, res = bj.bicgstab(h, Aloc, rhs, x, tol=1e-6, maxit=10000, comm=comm)
+        iters[0] = it
+        return res
+
+    for _ in range(args.warmup):
+        step()
+    barrier(ws)
+    sampler = ClockSampler(local)
+    bj.launch_count_reset()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    with sampler:
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        barrier(ws)
+        e0.record(stream)
+        for i in range(args.steps):
+            res = step(evs[i])
+        e1.record(stream)
+        barrier(ws)
+    torch.cuda.synchronize()
+    launches = bj.launch_count()
+    ms = max_over_ranks(e0.elapsed_time(e1), ws) / args.steps
+    setup_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
+    it = iters[0]
+    # SpMV alone (the dominant kernel): R27 over the local rows, CUDA events on its stream
+    nrep = 20
+    s0 = torch.cuda.Event(enable_timing=True)
+    s1 = torch.cuda.Event(enable_timing=True)
+    bj.spmv(Aloc, xs, ys)
+    s0.record(stream)
+    for _ in range(nrep):
+        bj.spmv(Aloc, xs, ys)
+    s1.record(stream)
+    torch.cuda.synchronize()
+    spmv_ms = s0.elapsed_time(s1) / nrep
+    spmv_bytes = 8 * (n + 1) + 12 * nnz + 16 * n          # row_ptr + (col, val) per entry + x read once + y write
+    achieved = spmv_bytes / (spmv_ms * 1e-3) / 1e9
+    solve_ms = ms - setup_ms
+    # per-iteration algorithmic bytes: 2 SpMV + 2 GETRS applies + vector updates / dots (16 vector passes)
+    m = sizes.long()
+    getrs_bytes = int((8 * m * m + 4 * m + 16 * m + 16).sum().item())
+    iter_bytes = 2 * spmv_bytes + 2 * getrs_bytes + 8 * n * (3 + 2 + 3 + 2 + 8)
+    line = {"metric": "preconditioned Krylov solves per second (setup + BiCGSTAB to 1e-6)",
+            "value": ws / (ms * 1e-3), "unit": "solves/s", "higher_is_better": True,
+            "n_gpus": ws, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic (counter-based FEM CSR generated on device)",
+            "config": {"workload": CONFIGS["C5K"][4], "block": b, "rows_per_gpu": n, "nnz_per_gpu": nnz,
+                       "iterations": it, "relative_residual": res, "l2": "CSR (1.9 GB/GPU) larger than L2"},
+            "breakdown_ms": {"setup": setup_ms, "solve": solve_ms, "per_iteration": solve_ms / max(it, 1),
+                             "spmv": spmv_ms},
+            "iteration_hbm": {"algorithmic_bytes": iter_bytes,
+                              "achieved_gbs": iter_bytes / (solve_ms / max(it, 1) * 1e-3) / 1e9},
+            "roofline": {"bound": "hbm", "kernel": "bj_spmv (k_spmv + k_spmv_long)", "achieved": achieved,
+                         "peak": hbm, "unit": "GB/s", "frac": achieved / hbm, "traffic": None,
+                         "peak_source": peak_src, "bytes_per_launch": spmv_bytes},
+            "gpu_launches": launches, "clocks": sampler.summary()}
+    if rank == 0 and ws == 1 and not args.no_cpu:
+        import time
+        import bj_synth as S
+        import oracle
+        rp, ci, va = S.fem_csr_fast(nx, ny, nz)
+        t0 = time.perf_counter()
+        _, it_o, res_o, *_ = oracle.bicgstab(rp, ci, va, S.uniform_block_ptr(n, b), np.ones(n))
+        t_o = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": 1.0 / t_o, "unit": "solves/s", "cores": os.cpu_count(), "kind": "oracle",
+                                "sample": f"one full solve incl. oracle extract + getrf ({it_o} iterations, "
+                                          f"same matrix); iterations equal: {it_o == it}"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
 def spawn(n: int) -> int:
     """`bench.py --gpus N` started as a plain process: re-launch it under
     torch.distributed.run with one rank per GPU (the launch the driver uses)."""
@@ -646,7 +763,9 @@ def main():
         run_reference(args, ws, rank)
         return
     ws, rank, local = dist_setup(args)
-    if args.config in FEM:
+    if args.config == "C5K":
+        run_krylov(args, ws, rank, local)
+    elif args.config in FEM:
         run_fem(args, ws, rank, local)
     else:
         run_ours(args, ws, rank, local)

@@ -40,7 +40,7 @@
 #include "internal.h"
 
 namespace bj {
-namespace {
+namespace krylov {
 
 constexpr int kChunk = 8192;        // R28: elements per chunk
 constexpr int kDotThreads = 256;    // R28: partial sums per chunk
@@ -64,83 +64,87 @@ struct Scalars {
 __device__ __forceinline__ double ld_stream(const double *p) { return __ldcs(p); }
 __device__ __forceinline__ int ld_stream(const int32_t *p) { return __ldcs(p); }
 
-// One pass of up to 4 entries per lane of two rows: issue every load first,
-// then the gathers, then the fma chains in entry order (lane l: entries
-// pass + l, + 32, + 64, + 96 of the row).  ra / rb = entries of the row left
-// from this lane's first entry of the pass (may be <= 0).
-__device__ __forceinline__ void spmv_pass2(const int32_t *__restrict__ ca, const double *__restrict__ va, int ra,
-                                           const int32_t *__restrict__ cb, const double *__restrict__ vb, int rb,
-                                           const double *__restrict__ x, double &s0, double &s1) {
-    int c[8];
-    double v[8], xv[8];
+// R27 with 8 lanes per row: lane lg of a row's group holds the lane
+// partials p = lg + 8q (q = 0..3).  Partial p accumulates the row's entries
+// p, p + 32, p + 64, ...; numbering the lane's entries lg + 8t (t = 0, 1, ...)
+// gives p = lg + 8 (t mod 4), and for a fixed q the slots t = q, q + 4, ...
+// come in increasing order -- the lane runs the four chains interleaved, each
+// in R27's order.  Butterfly: s_p += s_(p^16) and s_p += s_(p^8) are
+// in-lane adds (q^2, q^1); s_p += s_(p^4), (p^2), (p^1) are SHFL-xors inside
+// the group; y_i = s_0 = lane lg = 0, q = 0.
+constexpr int kGrp = 8;             // lanes per row
+constexpr int kSlots = 12;          // entries per lane per pass (96 per row)
+
+__device__ __forceinline__ double group_reduce(const double (&s)[4]) {
+    double u = (s[0] + s[2]) + (s[1] + s[3]);           // offsets 16 and 8
+    u = u + __shfl_xor_sync(0xffffffffu, u, 4);
+    u = u + __shfl_xor_sync(0xffffffffu, u, 2);
+    u = u + __shfl_xor_sync(0xffffffffu, u, 1);
+    return u;
+}
+
+// Rows of more than kLongRow entries (computed by k_spmv_long).
+__global__ void k_classify_long(int64_t n, const int64_t *__restrict__ rp, int32_t *long_rows, int32_t *nlong) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (rp[i + 1] - rp[i] > kLongRow) long_rows[atomicAdd(nlong, 1)] = (int32_t)i;
+}
+
+__global__ void __launch_bounds__(kSpmvThreads, 3) k_spmv(int64_t n, const int64_t *__restrict__ rp,
+                                                          const int32_t *__restrict__ ci,
+                                                          const double *__restrict__ val, int64_t coff,
+                                                          const double *__restrict__ x, double *__restrict__ y,
+                                                          const int *done) {
+    if (done && *done) return;
+    const int lane = threadIdx.x & 31, g = lane >> 3, lg = lane & 7;
+    const int64_t warp = (int64_t)blockIdx.x * (kSpmvThreads / 32) + (threadIdx.x >> 5);
+    const int64_t nwarps = (int64_t)gridDim.x * (kSpmvThreads / 32);
+    const int64_t ntask = (n + 31) / 32;
+    const double *xs = x - coff;                         // x indexed by the stored column id
+    for (int64_t task = warp; task < ntask; task += nwarps) {
+        const int64_t r0 = task * 32;
+        const int nr = (int)min((int64_t)32, n - r0);
+        const int64_t myp = rp[r0 + min(lane, nr - 1)];  // lane l: rp[r0 + l]
+        const int64_t lastp = rp[r0 + nr];
+        for (int k = 0; k < nr; k += 4) {
+            const int kr = k + g;                        // this group's row of the quad
+            const int64_t b = __shfl_sync(0xffffffffu, myp, kr & 31);
+            const int64_t e1 = __shfl_sync(0xffffffffu, myp, (kr + 1) & 31);
+            const int64_t e = (kr + 1 < nr) ? e1 : lastp;
+            int len = kr < nr ? (int)(e - b) : 0;
+            const bool skip = len > kLongRow;            // k_spmv_long's row
+            if (skip) len = 0;
+            const int maxlen = __reduce_max_sync(0xffffffffu, len);
+            const int32_t *cp = ci + b + lg;
+            const double *vp = val + b + lg;
+            const int rem = len - lg;                    // entries of this lane: offsets 8t < rem
+            double s[4] = {0.0, 0.0, 0.0, 0.0};
+            for (int base = 0; base < maxlen; base += kGrp * kSlots) {
+                int c[kSlots];
+                double v[kSlots], xv[kSlots];
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        c[q] = 0; v[q] = 0.0; c[4 + q] = 0; v[4 + q] = 0.0;
-        if (32 * q < ra) { c[q] = ld_stream(ca + 32 * q); v[q] = ld_stream(va + 32 * q); }
-        if (32 * q < rb) { c[4 + q] = ld_stream(cb + 32 * q); v[4 + q] = ld_stream(vb + 32 * q); }
-    }
+                for (int t = 0; t < kSlots; ++t) {
+                    const int o = base + 8 * t;
+                    c[t] = 0;
+                    v[t] = 0.0;
+                    if (o < rem) { c[t] = ld_stream(cp + o); v[t] = ld_stream(vp + o); }
+                }
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        xv[q] = 32 * q < ra ? x[c[q]] : 0.0;
-        xv[4 + q] = 32 * q < rb ? x[c[4 + q]] : 0.0;
-    }
+                for (int t = 0; t < kSlots; ++t) xv[t] = (base + 8 * t < rem) ? xs[c[t]] : 0.0;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        if (32 * q < ra) s0 = fma(v[q], xv[q], s0);
-        if (32 * q < rb) s1 = fma(v[4 + q], xv[4 + q], s1);
+                for (int t = 0; t < kSlots; ++t)
+                    if (base + 8 * t < rem) s[t & 3] = fma(v[t], xv[t], s[t & 3]);
+            }
+            const double u = group_reduce(s);
+            if (lg == 0 && kr < nr && !skip) y[r0 + kr] = u;
+        }
     }
 }
 
+// Full 32-lane butterfly of R27 (k_spmv_long: warp 0 holds s_l in lane l).
 __device__ __forceinline__ double butterfly(double s) {
 #pragma unroll
     for (int off = 16; off >= 1; off >>= 1) s = s + __shfl_xor_sync(0xffffffffu, s, off);
     return s;
-}
-
-__global__ void __launch_bounds__(kSpmvThreads, 3) k_spmv(int64_t n, const int64_t *__restrict__ rp,
-                                                       const int32_t *__restrict__ ci,
-                                                       const double *__restrict__ val, int64_t coff,
-                                                       const double *__restrict__ x, double *__restrict__ y,
-                                                       int32_t *long_rows, int32_t *nlong, const int *done) {
-    if (done && *done) return;
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = (int64_t)blockIdx.x * (kSpmvThreads / 32) + (threadIdx.x >> 5);
-    const int64_t nwarps = (int64_t)gridDim.x * (kSpmvThreads / 32);
-    const int64_t ntask = (n + 31) / 32;
-    for (int64_t task = warp; task < ntask; task += nwarps) {
-        const int64_t r0 = task * 32;
-        const int64_t nr = min((int64_t)32, n - r0);
-        // row pointers of the task: lane l holds rp[r0 + l]; rp[r0 + nr] by a broadcast load
-        const int64_t myp = rp[r0 + min((int64_t)lane, nr - 1)];
-        const int64_t lastp = rp[r0 + nr];
-        for (int k = 0; k < nr; k += 2) {
-            const int64_t b0 = __shfl_sync(0xffffffffu, myp, k);
-            const int64_t nx1 = __shfl_sync(0xffffffffu, myp, (k + 1) & 31);
-            const int64_t nx2 = __shfl_sync(0xffffffffu, myp, (k + 2) & 31);
-            const int64_t e0 = (k + 1 < nr) ? nx1 : lastp;
-            const int64_t b1 = e0;
-            const int64_t e1 = (k + 1 < nr) ? ((k + 2 < nr) ? nx2 : lastp) : e0;
-            // long rows go to k_spmv_long (queued once, by lane 0)
-            const bool long0 = e0 - b0 > kLongRow, long1 = e1 - b1 > kLongRow;
-            if (nlong && lane == 0) {
-                if (long0) long_rows[atomicAdd(nlong, 1)] = (int32_t)(r0 + k);
-                if (long1) long_rows[atomicAdd(nlong, 1)] = (int32_t)(r0 + k + 1);
-            }
-            const int l0 = long0 ? 0 : (int)(e0 - b0), l1 = long1 ? 0 : (int)(e1 - b1);
-            const int len = max(l0, l1);
-            double s0 = 0.0, s1 = 0.0;
-            const double *xs = x - coff;        // x indexed by global column
-            for (int pass = 0; pass < len; pass += 128)
-                spmv_pass2(ci + b0 + pass + lane, val + b0 + pass + lane, l0 - pass - lane,
-                           ci + b1 + pass + lane, val + b1 + pass + lane, l1 - pass - lane, xs, s0, s1);
-            s0 = butterfly(s0);
-            s1 = butterfly(s1);
-            if (lane == 0) {
-                if (!long0) y[r0 + k] = s0;
-                if (k + 1 < nr && !long1) y[r0 + k + 1] = s1;
-            }
-        }
-    }
 }
 
 // One CTA per long row (grid-stride over the queue).  Warp 0 owns the 32
@@ -334,21 +338,6 @@ __global__ void k_unpack(int64_t m, const double *__restrict__ src, double *__re
 
 enum Phase { kInit = 0, kAlpha = 1, kOmega = 2, kResid = 3, kDotOut = 4 };
 
-// Rank value of dot d: chunk partials added in chunk order from +0 (R28).
-__device__ double chunk_sum(const double *P, int64_t nc, int d) {
-    double acc = 0.0;
-    int64_t c = 0;
-    for (; c + 8 <= nc; c += 8) {
-        double t[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) t[u] = P[(c + u) * 4 + d];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) acc = acc + t[u];
-    }
-    for (; c < nc; ++c) acc = acc + P[c * 4 + d];
-    return acc;
-}
-
 // The scalar recurrences of R29 given the global dot values g[].
 __device__ void phase_apply(int phase, const double *g, Scalars *S, double *out) {
     switch (phase) {
@@ -390,16 +379,36 @@ __device__ void phase_apply(int phase, const double *g, Scalars *S, double *out)
     }
 }
 
-// Rank-local stage: chunk sums; with gather != nullptr they are published
-// for the caller's allgather, else the phase completes here (one rank).
-__global__ void k_phase_local(int phase, int nd, const double *P, int64_t nc, Scalars *S, double *gather,
-                              int rank, double *out) {
-    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+// Rank-local stage: chunk sums (R28: in chunk order from +0) -- the
+// partials are staged in shared memory by all threads (one round trip), then
+// one thread adds them in order.  With gather != nullptr the rank values are
+// published for the caller's allgather, else the phase completes here.
+constexpr int kPhaseThreads = 256;
+constexpr int kPhaseStage = 512;    // chunks staged per round
+__global__ void __launch_bounds__(kPhaseThreads) k_phase_local(int phase, int nd, const double *P, int64_t nc,
+                                                               Scalars *S, double *gather, int rank,
+                                                               double *out) {
     if (S && phase != kInit && S->done) return;
+    __shared__ double sp[kPhaseStage * 4];
     double g[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int d = 0; d < nd; ++d) g[d] = chunk_sum(P, nc, d);
+    for (int64_t c0 = 0; c0 < nc; c0 += kPhaseStage) {
+        const int cnt = (int)min((int64_t)kPhaseStage, nc - c0);
+        for (int i = threadIdx.x; i < cnt * 4; i += kPhaseThreads) sp[i] = P[c0 * 4 + i];
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int c = 0; c < cnt; ++c) {
+#pragma unroll
+                for (int d = 0; d < 4; ++d)
+                    if (d < nd) g[d] = g[d] + sp[c * 4 + d];
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x != 0) return;
     if (gather) {
-        for (int d = 0; d < nd; ++d) gather[rank * 4 + d] = g[d];
+#pragma unroll
+        for (int d = 0; d < 4; ++d)
+            if (d < nd) gather[rank * 4 + d] = g[d];
         return;
     }
     phase_apply(phase, g, S, out);
@@ -410,9 +419,11 @@ __global__ void k_phase_global(int phase, int nd, const double *gather, int nran
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     if (phase != kInit && S->done) return;
     double g[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int d = 0; d < nd; ++d) {
+#pragma unroll
+    for (int d = 0; d < 4; ++d) {
         double acc = 0.0;
-        for (int r = 0; r < nranks; ++r) acc = acc + gather[r * 4 + d];
+        if (d < nd)
+            for (int r = 0; r < nranks; ++r) acc = acc + gather[r * 4 + d];
         g[d] = acc;
     }
     phase_apply(phase, g, S, nullptr);
@@ -422,8 +433,16 @@ __global__ void k_phase_global(int phase, int nd, const double *gather, int nran
 
 int elem_grid() { return sm_count() * 8; }
 
-bj_status launch_spmv(const bj_csr &A, const double *x, double *y, int32_t *long_rows, int32_t *nlong,
-                      bool queue, const int *done, cudaStream_t s) {
+// Optional side stream for k_spmv_long: the few long rows run concurrently
+// with k_spmv (fork / join by events).
+struct LongCtx {
+    cudaStream_t side = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+};
+constexpr int kLongGrid = 32;
+
+bj_status launch_spmv(const bj_csr &A, const double *x, double *y, const int32_t *long_rows,
+                      const int32_t *nlong, const int *done, cudaStream_t s, const LongCtx *lc) {
     const int64_t n = A.nrows;
     if (n == 0) return BJ_OK;
     static int smem_set[64] = {0};
@@ -434,12 +453,29 @@ bj_status launch_spmv(const bj_csr &A, const double *x, double *y, int32_t *long
                                          (int)(4 * kSlice * sizeof(double))));
         smem_set[dev] = 1;
     }
-    const int grid = persistent_grid(k_spmv, kSpmvThreads);
-    k_spmv<<<grid, kSpmvThreads, 0, s>>>(n, A.row_ptr, A.col_idx, (const double *)A.values, A.col_offset, x, y,
-                                         long_rows, queue ? nlong : nullptr, done);
+    const double *vals = (const double *)A.values;
+    cudaStream_t ls = s;
+    if (lc) {
+        BJ_CUDA_TRY(cudaEventRecord(lc->fork, s));
+        BJ_CUDA_TRY(cudaStreamWaitEvent(lc->side, lc->fork, 0));
+        ls = lc->side;
+    }
+    k_spmv_long<<<kLongGrid, kLongThreads, 4 * kSlice * sizeof(double), ls>>>(A.row_ptr, A.col_idx, vals,
+                                                                              A.col_offset, x, y, long_rows,
+                                                                              nlong, done);
     BJ_LAUNCH_CHECK();
-    k_spmv_long<<<sm_count(), kLongThreads, 4 * kSlice * sizeof(double), s>>>(
-        A.row_ptr, A.col_idx, (const double *)A.values, A.col_offset, x, y, long_rows, nlong, done);
+    if (lc) BJ_CUDA_TRY(cudaEventRecord(lc->join, ls));
+    const int grid = persistent_grid(k_spmv, kSpmvThreads);
+    k_spmv<<<grid, kSpmvThreads, 0, s>>>(n, A.row_ptr, A.col_idx, vals, A.col_offset, x, y, done);
+    BJ_LAUNCH_CHECK();
+    if (lc) BJ_CUDA_TRY(cudaStreamWaitEvent(s, lc->join, 0));
+    return BJ_OK;
+}
+
+bj_status classify_long(const bj_csr &A, int32_t *long_rows, int32_t *nlong, cudaStream_t s) {
+    BJ_CUDA_TRY(cudaMemsetAsync(nlong, 0, sizeof(int32_t), s));
+    if (A.nrows == 0) return BJ_OK;
+    k_classify_long<<<elem_grid(), 256, 0, s>>>(A.nrows, A.row_ptr, long_rows, nlong);
     BJ_LAUNCH_CHECK();
     return BJ_OK;
 }
@@ -451,10 +487,11 @@ bj_status check_csr64(const bj_csr *A) {
     return BJ_OK;
 }
 
-}  // namespace
+}  // namespace krylov
 }  // namespace bj
 
 using namespace bj;
+using namespace bj::krylov;
 
 extern "C" bj_status bj_spmv(const bj_csr *A, const double *x, double *y, bj_stream_t stream) {
     bj_status st = check_csr64(A);
@@ -466,8 +503,21 @@ extern "C" bj_status bj_spmv(const bj_csr *A, const double *x, double *y, bj_str
     const int64_t cap = A->nnz / kLongRow + 2;
     BJ_CUDA_TRY(cudaMallocAsync((void **)&scr.p, (size_t)(cap + 1) * sizeof(int32_t), s));
     int32_t *nlong = (int32_t *)scr.p, *long_rows = nlong + 1;
-    BJ_CUDA_TRY(cudaMemsetAsync(nlong, 0, sizeof(int32_t), s));
-    return launch_spmv(*A, x, y, long_rows, nlong, true, nullptr, s);
+    if ((st = classify_long(*A, long_rows, nlong, s)) != BJ_OK) return st;
+    // per-device side stream + events for the long rows (created once, kept)
+    static LongCtx cached[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    LongCtx *lc = nullptr;
+    if (dev >= 0 && dev < 64) {
+        lc = &cached[dev];
+        if (!lc->side) {
+            BJ_CUDA_TRY(cudaStreamCreateWithFlags(&lc->side, cudaStreamNonBlocking));
+            BJ_CUDA_TRY(cudaEventCreateWithFlags(&lc->fork, cudaEventDisableTiming));
+            BJ_CUDA_TRY(cudaEventCreateWithFlags(&lc->join, cudaEventDisableTiming));
+        }
+    }
+    return launch_spmv(*A, x, y, long_rows, nlong, nullptr, s, lc);
 }
 
 extern "C" bj_status bj_dot(int64_t n, const double *x, const double *y, double *result, bj_stream_t stream) {
@@ -481,16 +531,17 @@ extern "C" bj_status bj_dot(int64_t n, const double *x, const double *y, double 
         k_dot<1><<<(unsigned)nc, kDotThreads, 0, s>>>(n, x, y, nullptr, nullptr, P, nullptr);
         BJ_LAUNCH_CHECK();
     }
-    k_phase_local<<<1, 32, 0, s>>>(kDotOut, 1, P, nc, nullptr, nullptr, 0, result);
+    k_phase_local<<<1, kPhaseThreads, 0, s>>>(kDotOut, 1, P, nc, nullptr, nullptr, 0, result);
     BJ_LAUNCH_CHECK();
     return BJ_OK;
 }
 
-namespace {
+namespace bj {
+namespace krylov {
 // dot phase: chunk partials already in P; completes the phase (comm or not)
 bj_status finish_phase(int phase, int nd, const double *P, int64_t nc, Scalars *S, const bj_comm *comm,
                        cudaStream_t s) {
-    k_phase_local<<<1, 32, 0, s>>>(phase, nd, P, nc, S, comm ? comm->gather_buf : nullptr,
+    k_phase_local<<<1, kPhaseThreads, 0, s>>>(phase, nd, P, nc, S, comm ? comm->gather_buf : nullptr,
                                    comm ? comm->rank : 0, nullptr);
     BJ_LAUNCH_CHECK();
     if (comm) {
@@ -514,7 +565,8 @@ bj_status halo(double *v, int64_t n, const bj_comm *comm, const int *done, cudaS
     }
     return BJ_OK;
 }
-}  // namespace
+}  // namespace krylov
+}  // namespace bj
 
 extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *comm, const double *b, double *x,
                                  double tol, int maxit, int *iters_h, double *resid_h, bj_stream_t stream) {
@@ -553,7 +605,7 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
     init.tol = tol;
     init.maxit = maxit;
     BJ_CUDA_TRY(cudaMemcpyAsync(S, &init, sizeof(Scalars), cudaMemcpyHostToDevice, s));
-    BJ_CUDA_TRY(cudaMemsetAsync(nlong, 0, sizeof(int32_t), s));
+    if ((st = classify_long(*A, long_rows, nlong, s)) != BJ_OK) return st;
     BJ_CUDA_TRY(cudaMemsetAsync(ph, 0, vecx, s));
     BJ_CUDA_TRY(cudaMemsetAsync(shv, 0, vecx, s));
     if (n > 0) {
@@ -570,20 +622,25 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
     BJ_CUDA_TRY(cudaHostAlloc((void **)&hflag, kRing * sizeof(int), cudaHostAllocDefault));
     cudaEvent_t ev[kRing];
     for (int i = 0; i < kRing; ++i) cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming);
+    LongCtx lc;
+    cudaStreamCreateWithFlags(&lc.side, cudaStreamNonBlocking);
+    cudaEventCreateWithFlags(&lc.fork, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&lc.join, cudaEventDisableTiming);
     auto cleanup = [&]() {
         for (int i = 0; i < kRing; ++i) cudaEventDestroy(ev[i]);
+        cudaEventDestroy(lc.fork);
+        cudaEventDestroy(lc.join);
+        cudaStreamDestroy(lc.side);
         cudaFreeHost(hflag);
     };
     const unsigned eg = (unsigned)elem_grid();
-    bool first_spmv = true;
     bj_status err = BJ_OK;
     for (int it = 1; it <= (maxit > 0 ? maxit : 0) && err == BJ_OK; ++it) {
         do {
             if (n > 0) { k_pupdate<<<eg, 256, 0, s>>>(n, S, p, v, r); BJ_LAUNCH_CHECK(); }
             if ((err = bj_apply(M, p, ph, stream)) != BJ_OK) break;
             if ((err = halo(ph, n, comm, done, s)) != BJ_OK) break;
-            if ((err = launch_spmv(*A, ph, v, long_rows, nlong, first_spmv, done, s)) != BJ_OK) break;
-            first_spmv = false;
+            if ((err = launch_spmv(*A, ph, v, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
             if (n > 0) {
                 k_dot<1><<<(unsigned)nc, kDotThreads, 0, s>>>(n, rh, v, nullptr, nullptr, P, done);
                 BJ_LAUNCH_CHECK();
@@ -592,7 +649,7 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
             if (n > 0) { k_supdate<<<eg, 256, 0, s>>>(n, S, sv, v, r); BJ_LAUNCH_CHECK(); }
             if ((err = bj_apply(M, sv, shv, stream)) != BJ_OK) break;
             if ((err = halo(shv, n, comm, done, s)) != BJ_OK) break;
-            if ((err = launch_spmv(*A, shv, t, long_rows, nlong, false, done, s)) != BJ_OK) break;
+            if ((err = launch_spmv(*A, shv, t, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
             if (n > 0) {
                 k_dot<2><<<(unsigned)nc, kDotThreads, 0, s>>>(n, t, sv, t, t, P, done);
                 BJ_LAUNCH_CHECK();
