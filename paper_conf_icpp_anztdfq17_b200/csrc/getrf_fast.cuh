@@ -51,6 +51,7 @@
 //    position tag-1 of every column and perm[tag-1] = r.
 #include "common.cuh"
 #include "internal.h"
+#include "getrs_tile.cuh"
 
 namespace bj {
 
@@ -76,10 +77,16 @@ template <> __device__ __forceinline__ bool fast_ok<float>(float x) {
 template <typename R> __host__ __device__ constexpr int panel_stride() { return sizeof(R) == 8 ? 34 : 36; }
 constexpr int kMaxPanel = 4;
 template <typename R>
-struct FastSmem {
+struct __align__(16) FastSmem {
     R row[32];                                    // pivot-row buffer, T elements per tile (sub-warp tiles)
     int pinv[32];                                 // fused solve: lane of the row at position k, per tile
     R panel[kMaxPanel][panel_stride<R>()];        // full-warp tiles: the panel's pivot rows (stale trailing part)
+};
+// bj_gesv_vbatched kernels of full-warp tiles: + the deferred-solve state
+template <typename R>
+struct __align__(16) FastSmemD : FastSmem<R> {     // 16-B multiple: the panel's STS.128 stay aligned
+    int64_t plo[4], pvo[4];                       // pending blocks (val_off, vec_off)
+    int keep;                                     // the last tile's block was kept (not sent to the safe path)
 };
 
 // Compile-time variants (scripts/micro/getrf_var.cu measures them):
@@ -493,7 +500,41 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
         piv[tk.vo + pos] = r;
     }
     if (keep && r == 0) info[blk] = __ffs((int)singmask);
-    if constexpr (SOLVE) getrf_tile_solve<R, M>(a, pos, row_keep, r, tbase, b + tk.vo, x + tk.vo, sm);
+    if constexpr (SOLVE) {
+        if constexpr (W32) {
+            // solved later by solve_pending (kernel loop); SOLVE && W32 only in FastSmemD kernels
+            if (lane == 0) static_cast<FastSmemD<R> &>(sm).keep = keep ? 1 : 0;
+        } else {
+            getrf_tile_solve<R, M>(a, pos, row_keep, r, tbase, b + tk.vo, x + tk.vo, sm);
+        }
+    }
+}
+
+// Deferred solve of bj_gesv_vbatched for full-warp tiles (M = 17..32): the
+// warp collects up to 4 blocks it has factored and kept (L\U and perm just
+// written, still in L2) and solves them together with the GETRS tile of
+// getrs_tile.cuh -- 8 lanes per block, 4 rows per lane -- reading the factors
+// back through L2 (coherent loads).  The SIMT solve from the registers
+// (getrf_tile_solve) costs every lane ~20 instructions per step for one FMA;
+// this costs the GETRS kernel's instructions and no HBM re-read.  Same
+// operations in the same order as GETRS: bit-identical.
+template <typename R, int M>
+__device__ __forceinline__ void solve_pending(const R *A, const int32_t *piv, const R *b, R *x,
+                                              const FastSmemD<R> &sm, int npend) {
+    constexpr int T = rs_lanes(M);
+    static_assert(T == 8, "full-warp GETRF tiles pair with 8-lane GETRS tiles");
+    const int lane = threadIdx.x & 31;
+    const int t = lane / T, q = lane % T;
+    const bool tile_ok = t < npend;
+    const int tt = tile_ok ? t : npend - 1;               // clamped: a valid block, store skipped
+    const int64_t lo = sm.plo[tt], vo = sm.pvo[tt];
+    int pv[4];
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+        const int rr = q + s * T;
+        pv[s] = rr < M ? __ldcg(piv + vo + rr) : 0;
+    }
+    getrs_rows<R, M, 6, true>(A + lo, piv + vo, b + vo, x + vo, tile_ok, q, pv);
 }
 
 // Out-of-line tile (kNoinline): each order gets its own register allocation
@@ -602,7 +643,10 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
              unsigned *__restrict__ safe_count, const R *b = nullptr, R *x = nullptr) {
     constexpr int NM = MHI - MLO + 1;
     __shared__ int64_t s_pref[NM + 1], s_first[NM], s_last[NM];
-    __shared__ __align__(16) FastSmem<R> s_warp[kFastThreads / 32];
+    // bj_gesv_vbatched on full-warp tiles: solves deferred in groups of 4 (solve_pending)
+    constexpr bool DEFER = SOLVE && MLO >= 17;
+    using Smem = std::conditional_t<DEFER, FastSmemD<R>, FastSmem<R>>;
+    __shared__ __align__(16) Smem s_warp[kFastThreads / 32];
     __shared__ __align__(128) R s_stage[kFastThreads / 32][stage_elems<R>(MLO, MHI)];
     constexpr int G = tiles_per_warp(MLO);
     __shared__ __align__(16) TaskRing<G> s_ring[kFastThreads / 32];
@@ -631,7 +675,8 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     __syncthreads();
     const int64_t ntask = s_pref[NM];
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    FastSmem<R> &sm = s_warp[w];
+    Smem &smd = s_warp[w];
+    FastSmem<R> &sm = smd;
     R *S = s_stage[w];
     TaskRing<G> &ring = s_ring[w];
     uint64_t *bar = &s_bar[w];
@@ -685,6 +730,8 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
     getrf_stage(A, slot_task(warp, 0), S, bar);
     unsigned parity = 0;
     int q0 = 0;
+    static_assert(!DEFER || MLO == MHI, "one order per full-warp kernel");
+    int npend = 0;
     for (int64_t task = warp; task < ntask; task += nwarps) {
         const int q1 = (q0 + 1) & 3, q2 = (q0 + 2) & 3, q3 = (q0 + 3) & 3;
         // ring: offsets of task+2 (its block id landed one iteration ago), block id of task+3
@@ -715,7 +762,27 @@ k_getrf_fast(R *A, const int64_t *__restrict__ val_off, const int64_t *__restric
         const StageNext<R> after_load{A, slot_task(task + nwarps, q1), S, bar};
         getrf_fast_dispatch<R, MLO, MHI, F, SOLVE>(A, cur, S, piv, info, safe_list, safe_count, b, x, sm,
                                                    after_load);
+        if constexpr (DEFER) {
+            __syncwarp();                            // sm.keep, L\U and perm of this task written
+            const bool kept = cur.ok && smd.keep != 0;
+            if (kept && lane == 0) {
+                smd.plo[npend] = cur.lo;
+                smd.pvo[npend] = cur.vo;
+            }
+            npend += kept ? 1 : 0;
+            if (npend == 4) {
+                __syncwarp();
+                solve_pending<R, MLO>(A, piv, b, x, smd, npend);
+                npend = 0;
+            }
+        }
         q0 = q1;
+    }
+    if constexpr (DEFER) {
+        if (npend > 0) {
+            __syncwarp();
+            solve_pending<R, MLO>(A, piv, b, x, smd, npend);
+        }
     }
     cp_async_wait_all();
     asm volatile("griddepcontrol.wait;" ::: "memory");

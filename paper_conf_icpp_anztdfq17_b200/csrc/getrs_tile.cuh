@@ -47,7 +47,16 @@ __device__ __noinline__ void getrs_slow_block(const R *LU, const int32_t *piv, c
 // Tiles past the end of the batch are given a valid block (the caller clamps
 // the index) and only skip the final store, so no load needs a tile predicate.
 // pv[s] = perm[q + s T] (prefetched by the caller, one task ahead).
-template <typename R, int M, int DR = 8>
+// Factor loads: read-only path (__ldg) when the factors come from an earlier
+// kernel; L2-coherent (__ldcg) when this kernel just wrote them (the deferred
+// solve of bj_gesv_vbatched, getrf_fast.cuh).
+template <bool COH, typename R>
+__device__ __forceinline__ R ld_factor(const R *p) {
+    if constexpr (COH) return __ldcg(p);
+    else return __ldg(p);
+}
+
+template <typename R, int M, int DR = 8, bool COH = false>
 __device__ __forceinline__ void getrs_rows(const R *__restrict__ LU, const int32_t *__restrict__ piv, const R *b,
                                            R *x, bool tile_ok, int q, const int (&pv)[4]) {
     constexpr int T = rs_lanes(M);
@@ -67,7 +76,7 @@ __device__ __forceinline__ void getrs_rows(const R *__restrict__ LU, const int32
         const int i = q + s * T;
         const bool ok = in_block(s, i);
         y[s] = ok ? b[pv[s]] : R(0);
-        dg[s] = ok ? __ldg(col + s * T + (int64_t)i * M) : R(1);
+        dg[s] = ok ? ld_factor<COH>(col + s * T + (int64_t)i * M) : R(1);
         yr[s] = Num<R>::rcp_refine(dg[s]);
     });
 
@@ -85,7 +94,7 @@ __device__ __forceinline__ void getrs_rows(const R *__restrict__ LU, const int32
             constexpr bool none = lower ? (s * T + T - 1 <= k) : (s * T >= k);
             if constexpr (!none) {
                 const int i = q + s * T;
-                ring[p % D][s] = in_block(s, i) ? __ldg(col + s * T + k * M) : R(0);
+                ring[p % D][s] = in_block(s, i) ? ld_factor<COH>(col + s * T + k * M) : R(0);
             }
         });
     };
