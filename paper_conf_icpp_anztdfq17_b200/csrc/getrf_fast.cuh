@@ -108,6 +108,14 @@ __host__ __device__ constexpr int panel_width(int F) {
 #ifndef BJ_FAST_DEFAULT
 #define BJ_FAST_DEFAULT 8
 #endif
+// Per-order flags of the single-order kernels (profiles/r02/
+// micro_getrf_flags_per_order.txt, 34.5k blocks per order): fp64 orders 25
+// and 27..32 spill at 128 registers (16 warps/SM); with 168 registers at 12
+// warps/SM they are 1-12 % faster.  kPre was slower for every order.
+template <typename R, int M>
+__host__ __device__ constexpr int fast_flags() {
+    return (sizeof(R) == 8 && M >= 25 && M != 26) ? (BJ_FAST_DEFAULT | kMin3) : BJ_FAST_DEFAULT;
+}
 // Resident CTAs (of 4 warps) per SM: explicit flags, else by the registers
 // the largest order of the class needs (row in registers + ~50).
 template <typename R>
@@ -793,7 +801,7 @@ template <typename R, int MLO, int MHI, bool SOLVE>
 bj_status launch_getrf_fast(R *A, const int64_t *val_off, const int64_t *vec_off, int32_t *piv, int32_t *info,
                             const PlanView &p, int32_t *safe_list, unsigned *safe_count, const R *b, R *x,
                             cudaStream_t s) {
-    auto kern = k_getrf_fast<R, MLO, MHI, BJ_FAST_DEFAULT, SOLVE>;
+    auto kern = k_getrf_fast<R, MLO, MHI, (MLO == MHI ? fast_flags<R, MLO>() : BJ_FAST_DEFAULT), SOLVE>;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(persistent_grid(kern, kFastThreads, true));
     cfg.blockDim = dim3(kFastThreads);

@@ -17,7 +17,7 @@
 namespace bj {
 
 template <typename R, int M>
-__global__ void __launch_bounds__(kFastThreads, fast_min_blocks<R>(BJ_FAST_DEFAULT, M))
+__global__ void __launch_bounds__(kFastThreads, fast_min_blocks<R>(fast_flags<R, M>(), M))
 k_setup_fused(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col_idx,
               const R *__restrict__ values, int64_t col_offset, const int32_t *__restrict__ block_ptr, R *A,
               const int64_t *__restrict__ val_off, const int64_t *__restrict__ vec_off, int32_t *__restrict__ piv,
@@ -60,7 +60,7 @@ k_setup_fused(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ c
         }
         extract_block_warp<R>(col_idx, values, col_offset, bs, M, rpv, e0, e1, S);
         auto nothing = [] {};
-        getrf_fast_tile<R, M, BJ_FAST_DEFAULT, false, decltype(nothing) &, true>(
+        getrf_fast_tile<R, M, fast_flags<R, M>(), false, decltype(nothing) &, true>(
             A, tk, S, piv, info, safe_list, safe_count, nullptr, nullptr, sm, nothing);
         __syncwarp();                        // the tile is read before the next extraction rewrites it
     }
