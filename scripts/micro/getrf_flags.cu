@@ -73,12 +73,19 @@ static Batch make(int64_t nb, int lo, int hi) {
 }
 
 
+#ifdef FLOAT
+using RT = float;
+#else
+using RT = double;
+#endif
 template <int M, int F>
 void run_order(int64_t nb) {
     Batch b = make(nb, M, M);
     int64_t tot = 0;
-    for (int64_t i = 0; i < nb; ++i) tot += (int64_t)(M * M + 1) / 2 * 2;
-    auto kern = k_getrf_fast<double, M, M, F>;
+    for (int64_t i = 0; i < nb; ++i) tot += (int64_t)(M * M + 3) / 4 * 4;
+    auto kern = k_getrf_fast<RT, M, M, F>;
+    RT *A = sizeof(RT) == 8 ? (RT *)b.A : (RT *)b.Af;
+    const RT *A0 = sizeof(RT) == 8 ? (const RT *)b.A0 : (const RT *)b.Af0;
     int per_sm = 0;
     cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFastThreads, 0);
@@ -86,18 +93,18 @@ void run_order(int64_t nb) {
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
     std::vector<float> ts;
     for (int rep = 0; rep < 8; ++rep) {
-        cudaMemcpy(b.A, b.A0, tot * 8, cudaMemcpyDeviceToDevice);
+        cudaMemcpy(A, A0, tot * sizeof(RT), cudaMemcpyDeviceToDevice);
         cudaMemset(b.cnt, 0, 4);
         cudaEventRecord(e0);
-        kern<<<grid, kFastThreads>>>(b.A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
+        kern<<<grid, kFastThreads>>>(A, b.dvo, b.dve, b.piv, b.info, b.dord, b.dbs, b.safe, b.cnt, nullptr, nullptr);
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms; cudaEventElapsedTime(&ms, e0, e1);
         if (rep > 1) ts.push_back(ms);
     }
     std::sort(ts.begin(), ts.end());
-    printf("M=%2d F=%3d occ=%2d warps/SM med %8.1f us min %8.1f us err=%s\n", M, F, per_sm * 4,
-           ts[ts.size() / 2] * 1e3, ts[0] * 1e3, cudaGetErrorString(cudaGetLastError()));
+    printf("%s M=%2d F=%3d occ=%2d warps/SM med %8.1f us min %8.1f us err=%s\n", sizeof(RT) == 8 ? "f64" : "f32", M, F,
+           per_sm * 4, ts[ts.size() / 2] * 1e3, ts[0] * 1e3, cudaGetErrorString(cudaGetLastError()));
     cudaFree(b.A); cudaFree(b.A0); cudaFree(b.Af); cudaFree(b.Af0);
 }
 template <int M>
