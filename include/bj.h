@@ -350,8 +350,13 @@ bj_status bj_halo_plan(int64_t nnz, const int32_t *col_idx_h, int64_t lo, int64_
  * and info_h (nblocks, may be NULL) back.  nvalues / nvec smaller than the
  * layout of sizes_h requires (sum of round_up(m^2, 16/s) / sum of m) is
  * BJ_ERR_ARG (checked on the host before any copy).
+ * Large batches (>= 131,072 blocks) run as up to 4 contiguous chunks in a
+ * pipeline: host-to-device copies (one copy stream), compute (`stream`) and
+ * device-to-host copies (a second copy stream) of different chunks overlap;
+ * results are identical to the unchunked call (the blocks are independent).
  * Device buffers live in `ws` and grow on demand.  Host buffers should be
- * pinned (cudaHostAlloc / torch pin_memory) for full PCIe bandwidth.
+ * pinned (cudaHostAlloc / torch pin_memory) for full PCIe bandwidth and for
+ * the copies to overlap.
  * ------------------------------------------------------------------------- */
 bj_status bj_workspace_create(bj_workspace **ws);
 bj_status bj_workspace_destroy(bj_workspace *ws);

@@ -1,7 +1,10 @@
 // api.cu -- the C ABI (include/bj.h): argument checking, plans, handles,
 // workspaces and dispatch to the kernel translation units.  No arithmetic of
 // the method lives here; there is no CPU or library fallback.
+#include <algorithm>
 #include <new>
+#include <vector>
+#include <stdlib.h>
 #include <string.h>
 
 #include "common.cuh"
@@ -439,17 +442,39 @@ bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int
         if (nvalues < need_val || nvec < need_vec) return BJ_ERR_ARG;
     }
     cudaStream_t s = (cudaStream_t)stream;
+    // Chunked pipeline: the batch is cut into K contiguous chunks; the copy
+    // engines move chunk c+1 in (stream sh) and chunk c-1 out (stream sd) while
+    // chunk c is factored and solved on the caller's stream, so PCIe time
+    // hides the compute.  Each chunk is an independent sub-batch (own layout
+    // and plan); the results are those of the whole batch (blocks are
+    // independent).
+    int K = (int)std::min<int64_t>(4, std::max<int64_t>(1, nb / 65536));
+    if (const char *ev_k = getenv("BJ_GESV_HOST_CHUNKS")) {     // experiment hook (bench / tests)
+        const int k = atoi(ev_k);
+        if (k >= 1 && k <= 64) K = (int)std::min<int64_t>(k, nb);
+    }
+    std::vector<int64_t> V(nb + 1), E(nb + 1), cb(K + 1);
+    {
+        const int64_t q = 16 / es;
+        V[0] = E[0] = 0;
+        for (int64_t i = 0; i < nb; ++i) {
+            const int64_t m = sizes_h[i] > 0 ? sizes_h[i] : 0;
+            V[i + 1] = V[i] + (m * m + q - 1) / q * q;
+            E[i + 1] = E[i] + m;
+        }
+        for (int c = 0; c <= K; ++c) cb[c] = nb * c / K;
+    }
     const size_t o_sizes = 0;
     const size_t o_vec = o_sizes + up256(sizeof(int32_t) * nb);
-    const size_t o_val = o_vec + up256(sizeof(int64_t) * (nb + 1));
-    const size_t o_A = o_val + up256(sizeof(int64_t) * (nb + 1));
+    const size_t o_val = o_vec + up256(sizeof(int64_t) * (nb + K));
+    const size_t o_A = o_val + up256(sizeof(int64_t) * (nb + K));
     const size_t o_b = o_A + up256((size_t)es * nvalues);
     const size_t o_x = o_b + up256((size_t)es * nvec);
     const size_t o_piv = o_x + up256((size_t)es * nvec);
     const size_t o_info = o_piv + up256(sizeof(int32_t) * nvec);
     const size_t o_order = o_info + up256(sizeof(int32_t) * nb);
     const size_t o_bins = o_order + up256(sizeof(int32_t) * nb);
-    const size_t need = o_bins + up256(sizeof(int64_t) * (kBins + 1));
+    const size_t need = o_bins + up256(sizeof(int64_t) * (kBins + 1) * K);
     if (need > ws->cap) {
         if (ws->dev) BJ_CUDA_TRY(cudaFree(ws->dev));
         ws->dev = nullptr;
@@ -461,26 +486,75 @@ bj_status bj_gesv_host(bj_workspace *ws, int64_t nb, const int32_t *sizes_h, int
     int32_t *sizes = (int32_t *)(d + o_sizes);
     int64_t *vec = (int64_t *)(d + o_vec), *val = (int64_t *)(d + o_val);
     int32_t *piv = (int32_t *)(d + o_piv), *info = (int32_t *)(d + o_info);
-    BJ_CUDA_TRY(cudaMemcpyAsync(sizes, sizes_h, sizeof(int32_t) * nb, cudaMemcpyHostToDevice, s));
-    BJ_CUDA_TRY(cudaMemcpyAsync(d + o_A, blocks_h, (size_t)es * nvalues, cudaMemcpyHostToDevice, s));
-    BJ_CUDA_TRY(cudaMemcpyAsync(d + o_b, b_h, (size_t)es * nvec, cudaMemcpyHostToDevice, s));
-    bj_status st;
-    if ((st = layout_sizes(nb, sizes, es, vec, val, s)) != BJ_OK) return st;
-    bj_plan p;
-    p.nblocks = nb;
-    p.order = (int32_t *)(d + o_order);
-    p.bin_start = (int64_t *)(d + o_bins);
-    if ((st = build_plan(nb, sizes, p.order, p.bin_start, s)) != BJ_OK) return st;
-    bj_batch batch{nb, sizes, vec, val, d + o_A, dtype};
-    // separate calls: measured faster than the fused bj_gesv_vbatched on B200
-    // (profiles/r02: the in-register solve costs more issue slots than
-    // re-reading the factors)
-    if ((st = bj_getrf_vbatched(&batch, piv, info, &p, stream)) != BJ_OK) return st;
-    if ((st = bj_getrs_vbatched(&batch, piv, d + o_b, d + o_x, &p, stream)) != BJ_OK) return st;
-    BJ_CUDA_TRY(cudaMemcpyAsync(x_h, d + o_x, (size_t)es * nvec, cudaMemcpyDeviceToHost, s));
-    if (pivots_h) BJ_CUDA_TRY(cudaMemcpyAsync(pivots_h, piv, sizeof(int32_t) * nvec, cudaMemcpyDeviceToHost, s));
-    if (info_h) BJ_CUDA_TRY(cudaMemcpyAsync(info_h, info, sizeof(int32_t) * nb, cudaMemcpyDeviceToHost, s));
-    BJ_CUDA_TRY(cudaStreamSynchronize(s));
+    char *A = d + o_A, *bd = d + o_b, *xd = d + o_x;
+    int32_t *order = (int32_t *)(d + o_order);
+    int64_t *bins = (int64_t *)(d + o_bins);
+    cudaStream_t sh = nullptr, sd = nullptr;
+    std::vector<cudaEvent_t> ev(2 * (size_t)K + 1, nullptr);
+    auto cleanup = [&]() {
+        if (sd) cudaStreamSynchronize(sd);
+        if (sh) cudaStreamSynchronize(sh);
+        cudaStreamSynchronize(s);
+        for (auto e : ev)
+            if (e) cudaEventDestroy(e);
+        if (sh) cudaStreamDestroy(sh);
+        if (sd) cudaStreamDestroy(sd);
+    };
+    bj_status st = BJ_OK;
+    do {
+        if (cudaStreamCreateWithFlags(&sh, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamCreateWithFlags(&sd, cudaStreamNonBlocking) != cudaSuccess) { st = BJ_ERR_CUDA; break; }
+        for (auto &e : ev)
+            if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { st = BJ_ERR_CUDA; break; }
+        if (st != BJ_OK) break;
+        // the workspace may still be in use by work the caller queued earlier on s
+        if (cudaEventRecord(ev[2 * K], s) != cudaSuccess || cudaStreamWaitEvent(sh, ev[2 * K], 0) != cudaSuccess) {
+            st = BJ_ERR_CUDA;
+            break;
+        }
+        const char *Ah = (const char *)blocks_h, *bh = (const char *)b_h;
+        for (int c = 0; c < K && st == BJ_OK; ++c) {          // inputs, chunk by chunk
+            const int64_t b0 = cb[c], b1 = cb[c + 1];
+            if (cudaMemcpyAsync(sizes + b0, sizes_h + b0, sizeof(int32_t) * (b1 - b0), cudaMemcpyHostToDevice, sh) ||
+                cudaMemcpyAsync(A + es * V[b0], Ah + es * V[b0], (size_t)es * (V[b1] - V[b0]), cudaMemcpyHostToDevice, sh) ||
+                cudaMemcpyAsync(bd + es * E[b0], bh + es * E[b0], (size_t)es * (E[b1] - E[b0]), cudaMemcpyHostToDevice, sh) ||
+                cudaEventRecord(ev[c], sh))
+                st = BJ_ERR_CUDA;
+        }
+        for (int c = 0; c < K && st == BJ_OK; ++c) {          // compute, chunk by chunk
+            const int64_t b0 = cb[c], b1 = cb[c + 1], n = b1 - b0;
+            if (n == 0) { if (cudaEventRecord(ev[K + c], s)) st = BJ_ERR_CUDA; continue; }
+            if (cudaStreamWaitEvent(s, ev[c], 0)) { st = BJ_ERR_CUDA; break; }
+            int64_t *vc = vec + b0 + c, *lc = val + b0 + c;
+            if ((st = layout_sizes(n, sizes + b0, es, vc, lc, s)) != BJ_OK) break;
+            bj_plan p;
+            p.nblocks = n;
+            p.order = order + b0;
+            p.bin_start = bins + (size_t)c * (kBins + 1);
+            if ((st = build_plan(n, sizes + b0, p.order, p.bin_start, s)) != BJ_OK) break;
+            bj_batch batch{n, sizes + b0, vc, lc, A + es * V[b0], dtype};
+            // separate calls: measured faster than the fused bj_gesv_vbatched on
+            // B200 (the solve is latency-bound)
+            if ((st = bj_getrf_vbatched(&batch, piv + E[b0], info + b0, &p, stream)) != BJ_OK) break;
+            if ((st = bj_getrs_vbatched(&batch, piv + E[b0], bd + es * E[b0], xd + es * E[b0], &p, stream)) != BJ_OK)
+                break;
+            if (cudaEventRecord(ev[K + c], s)) st = BJ_ERR_CUDA;
+        }
+        for (int c = 0; c < K && st == BJ_OK; ++c) {          // outputs, chunk by chunk
+            const int64_t b0 = cb[c], b1 = cb[c + 1];
+            if (cudaStreamWaitEvent(sd, ev[K + c], 0) ||
+                cudaMemcpyAsync((char *)x_h + es * E[b0], xd + es * E[b0], (size_t)es * (E[b1] - E[b0]),
+                                cudaMemcpyDeviceToHost, sd) ||
+                (pivots_h && cudaMemcpyAsync(pivots_h + E[b0], piv + E[b0], sizeof(int32_t) * (E[b1] - E[b0]),
+                                             cudaMemcpyDeviceToHost, sd)) ||
+                (info_h && cudaMemcpyAsync(info_h + b0, info + b0, sizeof(int32_t) * (b1 - b0),
+                                           cudaMemcpyDeviceToHost, sd)))
+                st = BJ_ERR_CUDA;
+        }
+    } while (0);
+    cleanup();
+    if (st != BJ_OK) return st;
+    if (cudaGetLastError() != cudaSuccess) return BJ_ERR_CUDA;
     return BJ_OK;
 }
 

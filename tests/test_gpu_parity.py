@@ -202,19 +202,23 @@ def test_device_generator_matches_host_generator():
                                                                                           dtype=NP[dtype])))
 
 
-def test_gesv_host_end_to_end():
-    """bj_gesv_host (host buffers in/out) equals the oracle."""
-    sizes = S.block_sizes(3000, 4, 32, first=7)
+@pytest.mark.parametrize("nb,pinned", [(3000, True), (300_001, True), (200_000, False)])
+def test_gesv_host_end_to_end(nb, pinned):
+    """bj_gesv_host (host buffers in/out) equals the oracle -- one chunk, and
+    the chunked copy/compute pipeline (nb >= 131,072: 4 and 3 chunks, ragged
+    chunk edges; pinned and pageable host buffers)."""
+    sizes = S.block_sizes(nb, 4, 32, first=7)
     vec, val = host_layout(sizes, torch.float64)
-    A = S.block_values(sizes, val, first=7)
+    A = S.block_values_fast(sizes, val, first=7) if nb > 3000 else S.block_values(sizes, val, first=7)
     b = S.rhs_values(sizes, first=7)
     ws = bj.Workspace()
-    sizes_h = torch.from_numpy(sizes).pin_memory()
-    A_h = torch.from_numpy(A).pin_memory()
-    b_h = torch.from_numpy(b).pin_memory()
-    x_h = torch.empty_like(b_h).pin_memory()
-    piv_h = torch.empty(int(vec[-1]), dtype=torch.int32).pin_memory()
-    info_h = torch.empty(len(sizes), dtype=torch.int32).pin_memory()
+    pin = (lambda t: t.pin_memory()) if pinned else (lambda t: t)
+    sizes_h = pin(torch.from_numpy(sizes))
+    A_h = pin(torch.from_numpy(A))
+    b_h = pin(torch.from_numpy(b))
+    x_h = pin(torch.empty_like(b_h))
+    piv_h = pin(torch.empty(int(vec[-1]), dtype=torch.int32))
+    info_h = pin(torch.empty(len(sizes), dtype=torch.int32))
     ws.gesv_host(sizes_h, A_h, b_h, x_h, piv_h, info_h)
     LU_o, piv_o, info_o = oracle.getrf_batch(sizes, val, vec, A)
     x_o = oracle.getrs_batch(sizes, val, vec, LU_o, piv_o, b)
