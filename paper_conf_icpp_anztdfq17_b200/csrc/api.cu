@@ -2,7 +2,9 @@
 // workspaces and dispatch to the kernel translation units.  No arithmetic of
 // the method lives here; there is no CPU or library fallback.
 #include <algorithm>
+#include <mutex>
 #include <new>
+#include <unordered_map>
 #include <vector>
 #include <stdlib.h>
 #include <string.h>
@@ -26,6 +28,31 @@ int sm_count() {
         cached[dev] = n > 0 ? n : 1;
     }
     return cached[dev];
+}
+
+// persistent_grid's cache (common.cuh): (kernel address, device, block size) -> grid
+namespace {
+struct GridKey {
+    const void *k;
+    int dev, threads;
+    bool operator==(const GridKey &o) const { return k == o.k && dev == o.dev && threads == o.threads; }
+};
+struct GridKeyHash {
+    size_t operator()(const GridKey &g) const {
+        return std::hash<const void *>()(g.k) ^ ((size_t)g.dev * 0x9E3779B97F4A7C15ull) ^ ((size_t)g.threads << 40);
+    }
+};
+std::mutex g_grid_mutex;
+std::unordered_map<GridKey, int, GridKeyHash> g_grid_cache;
+}  // namespace
+int grid_cache_get(const void *kernel, int dev, int threads) {
+    std::lock_guard<std::mutex> lock(g_grid_mutex);
+    auto it = g_grid_cache.find(GridKey{kernel, dev, threads});
+    return it == g_grid_cache.end() ? 0 : it->second;
+}
+void grid_cache_put(const void *kernel, int dev, int threads, int grid) {
+    std::lock_guard<std::mutex> lock(g_grid_mutex);
+    g_grid_cache[GridKey{kernel, dev, threads}] = grid;
 }
 
 static int elem_size(bj_dtype d) { return d == BJ_F64 ? 8 : d == BJ_F32 ? 4 : 0; }
