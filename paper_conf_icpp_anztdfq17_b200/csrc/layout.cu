@@ -81,28 +81,29 @@ k_plan_hist(const int32_t *__restrict__ sizes, int64_t n, int64_t *__restrict__ 
     for (int b = threadIdx.x; b < kBins; b += blockDim.x) hist[(int64_t)blockIdx.x * kBins + b] = cnt[b];
 }
 
-// Single CTA, one warp per bin: exclusive scan of hist[.][bin] over the tiles
-// (warp-wide chunks of 32), then bin starts; hist becomes the absolute start
-// of (tile, bin) in `order`.
+// Single CTA, one warp per bin.  Pass 1: bin totals (each lane sums a
+// strided subset of the tiles, warp reduction) -> bin starts.  Pass 2:
+// exclusive scan of hist[.][bin] over the tiles starting at the bin's start,
+// so hist becomes the absolute start of (tile, bin) in `order` directly.
 __global__ void __launch_bounds__(1024) k_plan_offsets(int64_t *hist, int64_t ntiles, int64_t *bin_start) {
     __shared__ int64_t tot[kBins];
     __shared__ int64_t base[kBins + 1];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     for (int b = w; b < kBins; b += nw) {
-        int64_t carry = 0;
-        for (int64_t t0 = 0; t0 < ntiles; t0 += 32) {
-            const int64_t t = t0 + lane;
-            const int64_t c = t < ntiles ? hist[t * kBins + b] : 0;
-            int64_t inc = c;
+        int64_t acc = 0;
+        for (int64_t T0 = 0; T0 < ntiles; T0 += 32 * 16) {    // 16 independent loads in flight per lane
+            int64_t cs[16];
 #pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const int64_t v = __shfl_up_sync(kFull, inc, off);
-                if (lane >= off) inc += v;
+            for (int j = 0; j < 16; ++j) {
+                const int64_t t = T0 + 32 * j + lane;
+                cs[j] = t < ntiles ? hist[t * kBins + b] : 0;
             }
-            if (t < ntiles) hist[t * kBins + b] = carry + inc - c;
-            carry += __shfl_sync(kFull, inc, 31);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) acc += cs[j];
         }
-        if (lane == 0) tot[b] = carry;
+#pragma unroll
+        for (int off = 16; off >= 1; off >>= 1) acc += __shfl_xor_sync(kFull, acc, off);
+        if (lane == 0) tot[b] = acc;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -115,7 +116,31 @@ __global__ void __launch_bounds__(1024) k_plan_offsets(int64_t *hist, int64_t nt
         bin_start[kBins] = s;
     }
     __syncthreads();
-    for (int64_t i = threadIdx.x; i < ntiles * kBins; i += blockDim.x) hist[i] += base[i % kBins];
+    constexpr int kAhead = 16;       // 32-tile chunks whose counts are loaded before the scans
+    for (int b = w; b < kBins; b += nw) {
+        int64_t carry = base[b];
+        for (int64_t T0 = 0; T0 < ntiles; T0 += 32 * kAhead) {
+            int64_t cs[kAhead];
+#pragma unroll
+            for (int j = 0; j < kAhead; ++j) {
+                const int64_t t = T0 + 32 * j + lane;
+                cs[j] = t < ntiles ? hist[t * kBins + b] : 0;
+            }
+#pragma unroll
+            for (int j = 0; j < kAhead; ++j) {
+                const int64_t t = T0 + 32 * j + lane;
+                const int64_t c = cs[j];
+                int64_t inc = c;
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const int64_t v = __shfl_up_sync(kFull, inc, off);
+                    if (lane >= off) inc += v;
+                }
+                if (t < ntiles) hist[t * kBins + b] = carry + inc - c;
+                carry += __shfl_sync(kFull, inc, 31);
+            }
+        }
+    }
 }
 
 __global__ void __launch_bounds__(kPlanThreads)

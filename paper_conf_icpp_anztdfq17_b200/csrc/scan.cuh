@@ -75,8 +75,13 @@ static __global__ void __launch_bounds__(kScanThreads) k_scan_partials(I64x2 *pa
 
 template <class F>
 __global__ void __launch_bounds__(kScanThreads) k_scan_down(F f, int64_t n, const I64x2 *partial) {
+    // Thread t scans items t*8 .. t*8+7 of the tile; the prefixes go through
+    // shared memory so the stores of vec/val are coalesced (consecutive
+    // threads -> consecutive items) instead of 8-element strided.
+    __shared__ long long oa[kScanTile], ob[kScanTile];
     I64x2 tot;
-    const int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanItems;
+    const int64_t tile0 = (int64_t)blockIdx.x * kScanTile;
+    const int64_t base = tile0 + (int64_t)threadIdx.x * kScanItems;
     I64x2 v[kScanItems];
     I64x2 s{0, 0};
 #pragma unroll
@@ -88,12 +93,15 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_down(F f, int64_t n, cons
     I64x2 ex = add2(block_exclusive_scan(s, tot), partial[blockIdx.x]);
 #pragma unroll
     for (int j = 0; j < kScanItems; ++j) {
-        int64_t i = base + j;
-        if (i < n) {
-            f.store(i, ex);
-            ex = add2(ex, v[j]);
-            if (i == n - 1) f.store(n, ex);
-        }
+        oa[threadIdx.x * kScanItems + j] = ex.a;
+        ob[threadIdx.x * kScanItems + j] = ex.b;
+        if (base + j == n - 1) f.store(n, add2(ex, v[j]));      // totals
+        ex = add2(ex, v[j]);
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < kScanTile; k += kScanThreads) {
+        const int64_t i = tile0 + k;
+        if (i < n) f.store(i, I64x2{oa[k], ob[k]});
     }
 }
 

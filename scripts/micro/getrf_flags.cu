@@ -110,7 +110,10 @@ void run_order(int64_t nb) {
 template <int M>
 void run_all() {
     run_order<M, FV>(34500);
-    if constexpr (M < 32) run_all<M + 1>();
+#ifndef MEND
+#define MEND 32
+#endif
+    if constexpr (M < MEND) run_all<M + 1>();
 }
 int main() {
     setvbuf(stdout, NULL, _IONBF, 0);
