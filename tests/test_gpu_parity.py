@@ -309,13 +309,13 @@ def test_c3_logical_sharding(G):
     torch.cuda.synchronize()
 
 
-def _gesv(sizes_np, dtype, kind="uniform", alias=False):
+def _gesv(sizes_np, dtype, kind="uniform", alias=False, values_np=None, b_np=None):
     """bj_gesv_vbatched (fused factor + solve) against the oracle's GETRF then
     GETRS, and against the library's own separate calls, bit for bit."""
     npdt = NP[dtype]
     vec, val = host_layout(sizes_np, dtype)
-    A = S.block_values(sizes_np, val, dtype=npdt, kind=kind)
-    b = S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt)
+    A = values_np if values_np is not None else S.block_values(sizes_np, val, dtype=npdt, kind=kind)
+    b = b_np if b_np is not None else S.rhs_values(np.maximum(sizes_np, 0), dtype=npdt)
     batch = device_batch(sizes_np, dtype, values_np=A)
     nvec = int(vec[-1])
     piv = torch.full((max(nvec, 1),), -7, dtype=torch.int32, device="cuda")
@@ -378,3 +378,41 @@ def test_gesv_c3_full_size_all_blocks():
     assert np.array_equal(piv.cpu().numpy(), piv_o)
     assert np.array_equal(bits(batch.values.cpu().numpy()[: len(LU_o)]), bits(LU_o))
     assert np.array_equal(bits(x.cpu().numpy()), bits(x_o))
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_advice_division_and_sign_of_zero_cases(dtype):
+    """The round-1 review's cases: a zero candidate divided by a subnormal or
+    an infinite pivot (L = 0, not NaN), GETRS with y_k = 0 over a subnormal /
+    infinite U(k,k), and an underflowing GER that would flip a -0 in a frozen
+    row (R3-R5) -- GETRF, GETRS and the fused GESV bit-identical
+    to the oracle, embedded in every tile width."""
+    npdt = NP[dtype]
+    sub = 1e-310 if dtype == torch.float64 else 1e-40
+    tiny = 1e-170 if dtype == torch.float64 else 1e-25
+    small = 1e-160 if dtype == torch.float64 else 1e-20
+    cases = [np.array([[sub, 1.0], [0.0, 1.0]]), np.array([[np.inf, 1.0], [0.0, 2.0]]),
+             np.array([[1.0, 0.0], [0.0, sub]]), np.array([[2.0, 1.0], [0.0, np.inf]]),
+             np.array([[1, 0, 0, tiny], [small, 1, 0, 0], [0, 0, 1, -1], [0, 0, 0.5, 1]], dtype=np.float64)]
+    blocks = []
+    for c in cases:
+        for m in (c.shape[0], 7, 16, 24, 32):           # alone and embedded (identity around it)
+            B = np.eye(m)
+            B[: c.shape[0], : c.shape[0]] = c
+            blocks.append(B)
+    sizes = np.array([B.shape[0] for B in blocks], np.int32)
+    vec, val = host_layout(sizes, dtype)
+    A = np.zeros(int(val[-1]), dtype=npdt)
+    b = np.zeros(int(vec[-1]), dtype=npdt)
+    for i, B in enumerate(blocks):
+        m = B.shape[0]
+        A[val[i]: val[i] + m * m] = B.astype(npdt).flatten(order="F")
+        rhs = np.zeros(m)
+        rhs[0] = 1.0                                     # y_1 = 0 over the special U(1,1)
+        b[vec[i]: vec[i] + m] = rhs.astype(npdt)
+    r = _run(sizes, dtype, values_np=A, b_np=b)
+    xd, xo = bits(r["x_d"]), bits(r["x_o"])
+    nan_d, nan_o = np.isnan(r["x_d"]), np.isnan(r["x_o"])
+    assert np.array_equal(nan_d, nan_o)
+    assert np.array_equal(xd[~nan_d], xo[~nan_o])
+    _gesv(sizes, dtype, values_np=A, b_np=b)
