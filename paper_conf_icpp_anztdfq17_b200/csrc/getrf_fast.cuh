@@ -35,16 +35,23 @@
 //        (pivoted rows, padding lanes, singular steps R4) use the multiplier
 //        +0, and fma(-0, u, a) == a bit for bit unless a == -0 (nvcc turns a
 //        predicated DFMA into DFMA + 2 FSEL, 5 instead of 3 issue slots per
-//        element).  No -0 can reach a frozen row: inputs hold none, SCAL
-//        writes only column k (never touched again) and a GER result is -0
-//        only through underflow.  Underflow is excluded by magnitudes: if
-//        every input and every final L\U entry is 0 or in [2^-450, 2^990)
-//        (fp32: [2^-39, 2^96); -0 allowed in the L part, which GER never
-//        touches after SCAL), every product l*u is 0 or >= 2^-900, a
-//        result below it in magnitude cannot cancel further, and every
-//        nonzero intermediate stays >= 2^-1006 (fp32 2^-126), above the
-//        subnormal range.  Blocks failing the input test go to k_getrf_safe
-//        at load time, blocks failing the output test are redone by it.
+//        element).  No -0 can reach a frozen row: inputs hold none (the
+//        input test), SCAL writes only column k (never touched again) and a
+//        GER result is -0 only through underflow.  Underflow and the fast
+//        quotient's domain are guarded by the OUTPUT test: every final L\U
+//        entry is 0 or in [2^-450, 2^990) (fp32: [2^-39, 2^96); -0 allowed
+//        in the L part, which GER never touches after SCAL).  Every product
+//        l*u of two outputs is then 0 or >= 2^-900 with granularity
+//        >= 2^-1004, so a GER result is exactly 0 (+0) or >= 2^-1005 in
+//        magnitude -- even when the other operand is a subnormal input,
+//        which a nonzero product swamps -- and never -0; a frozen row
+//        gains +-0 and keeps every value but -0 bit for bit.  A quotient is
+//        an output: a subnormal or huge dividend or pivot gives an output
+//        outside the range (the tile is redone).  Inf / NaN anywhere stay
+//        non-finite up to an output.  So the input test only has to reject
+//        -0 (one LOP3 + one min per element); blocks holding one go to
+//        k_getrf_safe at load time, blocks failing the output test are
+//        redone by it.
 //  * Partial pivoting grows entries by at most 2^31 in 32 steps, so every
 //    fast-path intermediate is finite.
 //  * Combined row swap at write-back: lane r stores its row at
@@ -57,8 +64,14 @@ namespace bj {
 
 constexpr int kFastThreads = 128;
 
-// Entries the fast path accepts, on input and in the final L\U (header
-// comment): +0, or |x| in [2^-450, 2^990) (fp32 [2^-39, 2^96)).  -0 and
+// Input test (header comment): 0 exactly for -0 (bits 0x8000...0).
+__device__ __forceinline__ unsigned neg_zero_key(double x) {
+    return ((unsigned)__double2hiint(x) ^ 0x80000000u) | (unsigned)__double2loint(x);
+}
+__device__ __forceinline__ unsigned neg_zero_key(float x) { return __float_as_uint(x) ^ 0x80000000u; }
+
+// Entries the fast path accepts in the final L\U (header comment): +0, or
+// |x| in [2^-450, 2^990) (fp32 [2^-39, 2^96)).  -0 (outside the L part) and
 // non-finite values fail.
 template <typename R> __device__ __forceinline__ bool fast_ok(R x);
 template <> __device__ __forceinline__ bool fast_ok<double>(double x) {
@@ -348,12 +361,13 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     R *Ab = A + tk.lo;
 
     R a[M];
-    bool ok = true;
+    unsigned nzmin = ~0u;                       // 0 iff the row holds a -0 (the input test)
     static_for<0, M>([&](auto jc) {
         constexpr int j = decltype(jc)::value;
         a[j] = (tile_ok && r < M) ? S[r + j * M] : R(0);
-        ok = ok && fast_ok(a[j]);
+        nzmin = min(nzmin, neg_zero_key(a[j]));
     });
+    const bool ok = nzmin != 0u;
     after_load();
     // Tiles with an entry outside the fast path's precondition go to the safe kernel.
     if (tile_bits<T>(__ballot_sync(kFull, !ok), tbase) != 0u) {
