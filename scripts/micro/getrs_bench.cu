@@ -79,5 +79,6 @@ int main() {
     run<17, 32>(40000, 32, 32, "C2 40k x 32");
     run<17, 32>(552000, 17, 32, "mix 17..32 552k");
     run<9, 16>(276000, 9, 16, "mix 9..16 276k");
+    run<17, 32>(83259, 24, 24, "C5 83k x 24");
     return 0;
 }
