@@ -201,3 +201,49 @@ def test_bicgstab_c5k_full_size():
     it, res = bj.bicgstab(h, A, torch.ones(n, dtype=torch.float64, device=DEV), x)
     assert it == it_o and res == res_o
     assert np.array_equal(bits(x.cpu().numpy()), bits(x_o))
+
+
+def test_bicgstab_torchcomm_nccl_one_rank():
+    """The multi-rank path with the real bj.TorchComm over NCCL (world size 1,
+    spawned in a fresh process): halo plan, callbacks issued from inside
+    bj_bicgstab, all_gather of the rank values -- bit-equal to the direct
+    single-GPU solve (R30 with one rank is R28)."""
+    import subprocess
+    import sys
+    import textwrap
+    code = textwrap.dedent("""
+        import os, socket, numpy as np, torch, torch.distributed as dist
+        import bj_synth as S
+        from paper_conf_icpp_anztdfq17_b200 import bj
+        s = socket.socket(); s.bind(("127.0.0.1", 0)); port = s.getsockname()[1]; s.close()
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        torch.cuda.set_device(0)
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+        g = S.FemGrid(10, 9, 8)
+        rp, ci, va = g.csr()
+        n = g.n
+        cl, hc, rc = bj.halo_plan(ci, 0, n, np.array([0, n], np.int64))
+        assert len(hc) == 0 and np.array_equal(cl, ci)
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+        A = bj.Csr(t(rp), t(ci), t(va), 0)
+        bp = t(S.uniform_block_ptr(n, 24))
+        sizes, vec, val = bj.layout_from_block_ptr(bp, torch.float64)
+        fac = bj.Batch(sizes, vec, val, torch.empty(int(val[-1].item()), dtype=torch.float64, device="cuda"))
+        piv = torch.empty(n, dtype=torch.int32, device="cuda")
+        info = torch.empty(bp.numel() - 1, dtype=torch.int32, device="cuda")
+        h = bj.Handle(); h.setup(A, bp, fac, piv, info)
+        b = torch.ones(n, dtype=torch.float64, device="cuda")
+        x0 = torch.empty(n, dtype=torch.float64, device="cuda")
+        it0, r0 = bj.bicgstab(h, A, b, x0)
+        comm = bj.TorchComm(hc, rc, 0, "cuda")
+        x1 = torch.empty(n, dtype=torch.float64, device="cuda")
+        it1, r1 = bj.bicgstab(h, A, b, x1, comm=comm)
+        assert it1 == it0 and r1 == r0, (it0, it1, r0, r1)
+        assert torch.equal(x0.view(torch.int64), x1.view(torch.int64))
+        dist.destroy_process_group()
+        print("torchcomm ok", it0)
+    """)
+    root = __import__("os").path.dirname(__import__("os").path.dirname(__import__("os").path.abspath(__file__)))
+    env = dict(__import__("os").environ, PYTHONPATH=root)
+    p = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True, text=True, timeout=300)
+    assert p.returncode == 0 and "torchcomm ok" in p.stdout, p.stdout[-2000:] + p.stderr[-4000:]
