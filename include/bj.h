@@ -305,7 +305,12 @@ bj_status bj_selftest_div(bj_dtype dtype, int64_t n, uint64_t seed, uint64_t *co
  *   and A->col_offset must be 0.  Before each SpMV the library packs
  *   x[send_idx[j]] into comm->send_buf and calls halo_exchange(ctx, stream),
  *   which must deliver every peer's entries into comm->recv_buf in halo order
- *   (stream-ordered).  For each dot the library writes its k <= 4 rank sums
+ *   (stream-ordered).  If halo_wait is not NULL the exchange may complete
+ *   asynchronously: the library then computes the INTERIOR rows (no halo
+ *   column) while it is in flight, calls halo_wait(ctx, stream) -- after
+ *   which recv_buf must be complete in stream order -- and computes the
+ *   boundary rows (each row's value is the same R27 result either way).
+ *   For each dot the library writes its k <= 4 rank sums
  *   to gather_buf[rank*4 .. rank*4+k) and calls allgather(ctx, k, stream),
  *   which must fill every rank's row; the global value is the sum over ranks
  *   in rank order from +0 (reading R30; one rank reproduces R28 exactly).
@@ -332,6 +337,7 @@ typedef struct {
     double *gather_buf;         /* device [nranks * 4], caller-owned            */
     int (*halo_exchange)(void *ctx, bj_stream_t stream);
     int (*allgather)(void *ctx, int k, bj_stream_t stream);
+    int (*halo_wait)(void *ctx, bj_stream_t stream);   /* optional (NULL: exchange is stream-synchronous) */
 } bj_comm;
 
 bj_status bj_spmv(const bj_csr *A, const double *x, double *y, bj_stream_t stream);

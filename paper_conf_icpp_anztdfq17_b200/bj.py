@@ -52,7 +52,7 @@ class CommC(ctypes.Structure):
     _fields_ = [("ctx", ctypes.c_void_p), ("nranks", ctypes.c_int), ("rank", ctypes.c_int),
                 ("nhalo", ctypes.c_int64), ("nsend", ctypes.c_int64), ("send_idx", ctypes.c_void_p),
                 ("send_buf", ctypes.c_void_p), ("recv_buf", ctypes.c_void_p), ("gather_buf", ctypes.c_void_p),
-                ("halo_exchange", HALO_FN), ("allgather", GATHER_FN)]
+                ("halo_exchange", HALO_FN), ("allgather", GATHER_FN), ("halo_wait", HALO_FN)]
 
 
 class BatchC(ctypes.Structure):
@@ -477,12 +477,21 @@ class TorchComm:
         self.nsend, self.nhalo = want.numel(), req.numel()
         self._halo_cb = HALO_FN(self._halo)
         self._gather_cb = GATHER_FN(self._gather)
+        self._wait_cb = HALO_FN(self._wait)
 
-    def halo_exchange(self):
-        """send_buf -> recv_buf (grouped by owner rank, halo order)."""
-        self.dist.all_to_all_single(self.recv_buf[: self.nhalo], self.send_buf[: self.nsend],
-                                    output_split_sizes=self.recv_counts, input_split_sizes=self.send_counts,
-                                    group=self.group)
+    def halo_exchange(self, async_op: bool = False):
+        """send_buf -> recv_buf (grouped by owner rank, halo order).  With
+        async_op the exchange is left in flight until halo_wait()."""
+        self._work = self.dist.all_to_all_single(self.recv_buf[: self.nhalo], self.send_buf[: self.nsend],
+                                                 output_split_sizes=self.recv_counts,
+                                                 input_split_sizes=self.send_counts, group=self.group,
+                                                 async_op=async_op)
+
+    def halo_wait(self):
+        """make the current stream wait for the exchange started by halo_exchange(async_op=True)."""
+        w, self._work = getattr(self, "_work", None), None
+        if w is not None:
+            w.wait()
 
     def allgather(self, k: int):
         """every rank's row gather_buf[r*4 : r*4+4] to every rank."""
@@ -491,7 +500,14 @@ class TorchComm:
 
     def _halo(self, ctx, stream):
         try:
-            self.halo_exchange()
+            self.halo_exchange(async_op=True)     # the library computes the interior rows meanwhile
+            return 0
+        except Exception:
+            return 1
+
+    def _wait(self, ctx, stream):
+        try:
+            self.halo_wait()
             return 0
         except Exception:
             return 1
@@ -505,7 +521,7 @@ class TorchComm:
 
     def c(self) -> CommC:
         return CommC(None, self.nranks, self.rank, self.nhalo, self.nsend, _p(self.send_idx), _p(self.send_buf),
-                     _p(self.recv_buf), _p(self.gather_buf), self._halo_cb, self._gather_cb)
+                     _p(self.recv_buf), _p(self.gather_buf), self._halo_cb, self._gather_cb, self._wait_cb)
 
 
 class LoopbackComm(TorchComm):
@@ -519,12 +535,16 @@ class LoopbackComm(TorchComm):
         self.recv_buf = torch.zeros(1, dtype=torch.float64, device=self.device)
         self.gather_buf = torch.zeros(4, dtype=torch.float64, device=self.device)
         self.nsend = self.nhalo = 0
-        self.calls = {"halo": 0, "allgather": 0}
+        self.calls = {"halo": 0, "allgather": 0, "wait": 0}
         self._halo_cb = HALO_FN(self._halo)
         self._gather_cb = GATHER_FN(self._gather)
+        self._wait_cb = HALO_FN(self._wait)
 
-    def halo_exchange(self):
+    def halo_exchange(self, async_op: bool = False):
         self.calls["halo"] += 1
+
+    def halo_wait(self):
+        self.calls["wait"] += 1
 
     def allgather(self, k: int):
         self.calls["allgather"] += 1

@@ -140,6 +140,78 @@ __global__ void __launch_bounds__(kSpmvThreads, 3) k_spmv(int64_t n, const int64
     }
 }
 
+// k_spmv over an explicit list of rows (multi-rank solves: interior rows
+// while the halo is in flight, then the boundary rows).  Same per-row code
+// and order as k_spmv; tasks of 32 listed rows, row pointers per lane.
+__global__ void __launch_bounds__(kSpmvThreads, 3) k_spmv_rows(int64_t nlist, const int32_t *__restrict__ list,
+                                                               const int64_t *__restrict__ rp,
+                                                               const int32_t *__restrict__ ci,
+                                                               const double *__restrict__ val,
+                                                               const double *__restrict__ x,
+                                                               double *__restrict__ y, const int *done) {
+    if (done && *done) return;
+    const int lane = threadIdx.x & 31, g = lane >> 3, lg = lane & 7;
+    const int64_t warp = (int64_t)blockIdx.x * (kSpmvThreads / 32) + (threadIdx.x >> 5);
+    const int64_t nwarps = (int64_t)gridDim.x * (kSpmvThreads / 32);
+    const int64_t ntask = (nlist + 31) / 32;
+    for (int64_t task = warp; task < ntask; task += nwarps) {
+        const int64_t t0 = task * 32;
+        const int nr = (int)min((int64_t)32, nlist - t0);
+        const int myrow = list[t0 + min(lane, nr - 1)];
+        const int64_t myb = rp[myrow], mye = rp[myrow + 1];
+        for (int k = 0; k < nr; k += 4) {
+            const int kr = k + g;
+            const int row = __shfl_sync(0xffffffffu, myrow, kr & 31);
+            const int64_t b = __shfl_sync(0xffffffffu, myb, kr & 31);
+            const int64_t e = __shfl_sync(0xffffffffu, mye, kr & 31);
+            int len = kr < nr ? (int)(e - b) : 0;
+            const bool skip = len > kLongRow;            // k_spmv_long's row
+            if (skip) len = 0;
+            const int maxlen = __reduce_max_sync(0xffffffffu, len);
+            const int32_t *cp = ci + b + lg;
+            const double *vp = val + b + lg;
+            const int rem = len - lg;
+            double s[4] = {0.0, 0.0, 0.0, 0.0};
+            for (int base = 0; base < maxlen; base += kGrp * kSlots) {
+                int c[kSlots];
+                double v[kSlots], xv[kSlots];
+#pragma unroll
+                for (int t = 0; t < kSlots; ++t) {
+                    const int o = base + 8 * t;
+                    c[t] = 0;
+                    v[t] = 0.0;
+                    if (o < rem) { c[t] = ld_stream(cp + o); v[t] = ld_stream(vp + o); }
+                }
+#pragma unroll
+                for (int t = 0; t < kSlots; ++t) xv[t] = (base + 8 * t < rem) ? x[c[t]] : 0.0;
+#pragma unroll
+                for (int t = 0; t < kSlots; ++t)
+                    if (base + 8 * t < rem) s[t & 3] = fma(v[t], xv[t], s[t & 3]);
+            }
+            const double u = group_reduce(s);
+            if (lg == 0 && kr < nr && !skip) y[row] = u;
+        }
+    }
+}
+
+// Rows with a halo column (local extended id >= n) -> boundary list, the
+// others -> interior list (warp per row; append order is irrelevant).
+__global__ void k_split_rows(int64_t n, const int64_t *__restrict__ rp, const int32_t *__restrict__ ci,
+                             int32_t *interior, int32_t *ninterior, int32_t *boundary, int32_t *nboundary) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = warp; i < n; i += nwarps) {
+        bool remote = false;
+        for (int64_t e = rp[i] + lane; e < rp[i + 1]; e += 32) remote = remote || ci[e] >= n;
+        remote = __any_sync(0xffffffffu, remote);
+        if (lane == 0) {
+            if (remote) boundary[atomicAdd(nboundary, 1)] = (int32_t)i;
+            else interior[atomicAdd(ninterior, 1)] = (int32_t)i;
+        }
+    }
+}
+
 // Full 32-lane butterfly of R27 (k_spmv_long: warp 0 holds s_l in lane l).
 __device__ __forceinline__ double butterfly(double s) {
 #pragma unroll
@@ -552,17 +624,53 @@ bj_status finish_phase(int phase, int nd, const double *P, int64_t nc, Scalars *
     return BJ_OK;
 }
 
-bj_status halo(double *v, int64_t n, const bj_comm *comm, const int *done, cudaStream_t s) {
-    if (!comm) return BJ_OK;
+struct RowLists {
+    int32_t *interior = nullptr, *boundary = nullptr;
+    int64_t ninterior = 0, nboundary = 0;
+};
+
+// Multi-rank SpMV (R27 per row, R30 solve): pack the rows peers need, start
+// the halo exchange, compute the interior rows while it is in flight (when
+// the caller provides halo_wait), complete it, unpack the halo behind the
+// own rows of v, compute the boundary rows, then the long rows (which may
+// touch the halo).
+bj_status spmv_comm(const bj_csr &A, double *v, double *y, const bj_comm *comm, const RowLists &rl,
+                    const int32_t *long_rows, const int32_t *nlong, const int *done, cudaStream_t s) {
+    const int64_t n = A.nrows;
+    const double *vals = (const double *)A.values;
+    const int grid = persistent_grid(k_spmv_rows, kSpmvThreads);
     if (comm->nsend > 0) {
         k_pack<<<elem_grid(), 256, 0, s>>>(comm->nsend, comm->send_idx, v, comm->send_buf, done);
         BJ_LAUNCH_CHECK();
     }
     if (comm->halo_exchange(comm->ctx, (bj_stream_t)s) != 0) return BJ_ERR_COMM;
+    auto rows = [&](const int32_t *list, int64_t cnt) -> bj_status {
+        if (cnt == 0) return BJ_OK;
+        k_spmv_rows<<<grid, kSpmvThreads, 0, s>>>(cnt, list, A.row_ptr, A.col_idx, vals, v, y, done);
+        BJ_LAUNCH_CHECK();
+        return BJ_OK;
+    };
+    bj_status st;
+    const bool overlap = comm->halo_wait != nullptr;
+    if (overlap && (st = rows(rl.interior, rl.ninterior)) != BJ_OK) return st;
+    if (overlap && comm->halo_wait(comm->ctx, (bj_stream_t)s) != 0) return BJ_ERR_COMM;
     if (comm->nhalo > 0) {
         k_unpack<<<elem_grid(), 256, 0, s>>>(comm->nhalo, comm->recv_buf, v + n, done);
         BJ_LAUNCH_CHECK();
     }
+    if (!overlap && (st = rows(rl.interior, rl.ninterior)) != BJ_OK) return st;
+    if ((st = rows(rl.boundary, rl.nboundary)) != BJ_OK) return st;
+    static int smem_set[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !smem_set[dev]) {
+        BJ_CUDA_TRY(cudaFuncSetAttribute(k_spmv_long, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(4 * kSlice * sizeof(double))));
+        smem_set[dev] = 1;
+    }
+    k_spmv_long<<<kLongGrid, kLongThreads, 4 * kSlice * sizeof(double), s>>>(A.row_ptr, A.col_idx, vals, 0, v, y,
+                                                                              long_rows, nlong, done);
+    BJ_LAUNCH_CHECK();
     return BJ_OK;
 }
 }  // namespace krylov
@@ -589,7 +697,8 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
     const size_t o_r = 0, o_rh = o_r + up(vec), o_p = o_rh + up(vec), o_v = o_p + up(vec), o_s = o_v + up(vec),
                  o_t = o_s + up(vec), o_ph = o_t + up(vec), o_sh = o_ph + up(vecx), o_P = o_sh + up(vecx),
                  o_S = o_P + up((size_t)(nc > 0 ? nc : 1) * 32), o_q = o_S + up(sizeof(Scalars)),
-                 total = o_q + up((size_t)(cap + 1) * 4);
+                 o_lists = o_q + up((size_t)(cap + 1) * 4),
+                 total = o_lists + (comm ? up((size_t)(2 * (n > 0 ? n : 1) + 2) * 4) : 0);
     AsyncScratch scr(s);
     BJ_CUDA_TRY(cudaMallocAsync((void **)&scr.p, total, s));
     char *base = scr.p;
@@ -598,6 +707,7 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
            *ph = (double *)(base + o_ph), *shv = (double *)(base + o_sh), *P = (double *)(base + o_P);
     Scalars *S = (Scalars *)(base + o_S);
     int32_t *nlong = (int32_t *)(base + o_q), *long_rows = nlong + 1;
+    RowLists rl{};
     const int *done = &S->done;
 
     // initial state; x0 = 0 also defines the halo parts of ph / sh (never read before written)
@@ -606,6 +716,19 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
     init.maxit = maxit;
     BJ_CUDA_TRY(cudaMemcpyAsync(S, &init, sizeof(Scalars), cudaMemcpyHostToDevice, s));
     if ((st = classify_long(*A, long_rows, nlong, s)) != BJ_OK) return st;
+    if (comm && n > 0) {   // interior / boundary rows (counts to the host once)
+        int32_t *cnt = (int32_t *)(base + o_lists);
+        rl.interior = cnt + 2;
+        rl.boundary = rl.interior + n;
+        BJ_CUDA_TRY(cudaMemsetAsync(cnt, 0, 2 * sizeof(int32_t), s));
+        k_split_rows<<<elem_grid(), 256, 0, s>>>(n, A->row_ptr, A->col_idx, rl.interior, cnt, rl.boundary, cnt + 1);
+        BJ_LAUNCH_CHECK();
+        int32_t hc[2] = {0, 0};
+        BJ_CUDA_TRY(cudaMemcpyAsync(hc, cnt, sizeof(hc), cudaMemcpyDeviceToHost, s));
+        BJ_CUDA_TRY(cudaStreamSynchronize(s));
+        rl.ninterior = hc[0];
+        rl.nboundary = hc[1];
+    }
     BJ_CUDA_TRY(cudaMemsetAsync(ph, 0, vecx, s));
     BJ_CUDA_TRY(cudaMemsetAsync(shv, 0, vecx, s));
     if (n > 0) {
@@ -639,8 +762,8 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
         do {
             if (n > 0) { k_pupdate<<<eg, 256, 0, s>>>(n, S, p, v, r); BJ_LAUNCH_CHECK(); }
             if ((err = bj_apply(M, p, ph, stream)) != BJ_OK) break;
-            if ((err = halo(ph, n, comm, done, s)) != BJ_OK) break;
-            if ((err = launch_spmv(*A, ph, v, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
+            if ((err = comm ? spmv_comm(*A, ph, v, comm, rl, long_rows, nlong, done, s)
+                            : launch_spmv(*A, ph, v, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
             if (n > 0) {
                 k_dot<1><<<(unsigned)nc, kDotThreads, 0, s>>>(n, rh, v, nullptr, nullptr, P, done);
                 BJ_LAUNCH_CHECK();
@@ -648,8 +771,8 @@ extern "C" bj_status bj_bicgstab(bj_handle *M, const bj_csr *A, const bj_comm *c
             if ((err = finish_phase(kAlpha, 1, P, nc, S, comm, s)) != BJ_OK) break;
             if (n > 0) { k_supdate<<<eg, 256, 0, s>>>(n, S, sv, v, r); BJ_LAUNCH_CHECK(); }
             if ((err = bj_apply(M, sv, shv, stream)) != BJ_OK) break;
-            if ((err = halo(shv, n, comm, done, s)) != BJ_OK) break;
-            if ((err = launch_spmv(*A, shv, t, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
+            if ((err = comm ? spmv_comm(*A, shv, t, comm, rl, long_rows, nlong, done, s)
+                            : launch_spmv(*A, shv, t, long_rows, nlong, done, s, &lc)) != BJ_OK) break;
             if (n > 0) {
                 k_dot<2><<<(unsigned)nc, kDotThreads, 0, s>>>(n, t, sv, t, t, P, done);
                 BJ_LAUNCH_CHECK();

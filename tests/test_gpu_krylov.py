@@ -162,6 +162,7 @@ def test_bicgstab_loopback_comm_path_equal():
     x1, it1, res1 = _solve_both(rp, ci, va, bp, b, comm=comm)
     assert it1 == it0 and res1 == res0 and np.array_equal(bits(x1), bits(x0))
     assert comm.calls["halo"] >= 2 * it0 and comm.calls["allgather"] >= 3 * it0 + 1
+    assert comm.calls["wait"] == comm.calls["halo"]
 
 
 def test_bicgstab_inverse_handle_converges():
