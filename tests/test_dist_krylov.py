@@ -78,7 +78,8 @@ def _worker(rank, world, port, q):
             ext = np.zeros(n + nh)
             ext[:n] = u
             comm.send_buf[: comm.nsend] = torch.from_numpy(u[comm.send_idx.numpy()])
-            comm.halo_exchange()
+            comm.halo_exchange(async_op=True)      # the library's order: start, (interior rows), wait
+            comm.halo_wait()
             ext[n:] = comm.recv_buf[:nh].numpy()
             return ext
 
