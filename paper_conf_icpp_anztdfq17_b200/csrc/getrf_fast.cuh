@@ -70,6 +70,17 @@ __device__ __forceinline__ unsigned neg_zero_key(double x) {
 }
 __device__ __forceinline__ unsigned neg_zero_key(float x) { return __float_as_uint(x) ^ 0x80000000u; }
 
+// Output test with kOut2: +-0 or |x| in [2^-450, 2^990) (fp32 [2^-39, 2^96)).
+template <typename R> __device__ __forceinline__ bool fast_ok_out(R x);
+template <> __device__ __forceinline__ bool fast_ok_out<double>(double x) {
+    const unsigned h = (unsigned)__double2hiint(x) & 0x7fffffffu, lo = (unsigned)__double2loint(x);
+    return (h - 0x23D00000u < 0x7DD00000u - 0x23D00000u) || ((h | lo) == 0u);
+}
+template <> __device__ __forceinline__ bool fast_ok_out<float>(float x) {
+    const unsigned b = __float_as_uint(x) & 0x7fffffffu;
+    return (b - (88u << 23) < (223u << 23) - (88u << 23)) || b == 0u;
+}
+
 // Entries the fast path accepts in the final L\U (header comment): +0, or
 // |x| in [2^-450, 2^990) (fp32 [2^-39, 2^96)).  -0 (outside the L part) and
 // non-finite values fail.
@@ -113,8 +124,11 @@ struct __align__(16) FastSmemD : FastSmem<R> {     // 16-B multiple: the panel's
 //   kMin5 / kMin6 -- 5 / 6 CTAs (20 / 24 warps) per SM (102 / 85 registers).
 //   kMin4 -- 4 CTAs (16 warps) per SM (128 registers).
 //   kNoinline -- per-order tiles out of line (one launch per order range).
+//   kOut2 -- output test without the L-part position check (a -0 can only
+//            be an L entry, header comment); changes the register allocation,
+//            so it is chosen per order (micro_getrf_flags_per_order.txt).
 constexpr int kPre = 1, kMin3 = 2, kVol = 4, kPanel2 = 8, kPanel3 = 16, kPanel4 = 32, kMin5 = 64, kMin6 = 128,
-              kMin4 = 256, kNoinline = 512;
+              kMin4 = 256, kNoinline = 512, kOut2 = 1024;
 __host__ __device__ constexpr int panel_width(int F) {
     return (F & kPanel4) ? 4 : (F & kPanel3) ? 3 : (F & kPanel2) ? 2 : 1;
 }
@@ -127,7 +141,9 @@ __host__ __device__ constexpr int panel_width(int F) {
 // warps/SM they are 1-12 % faster.  kPre was slower for every order.
 template <typename R, int M>
 __host__ __device__ constexpr int fast_flags() {
-    return (sizeof(R) == 8 && M >= 25 && M != 26) ? (BJ_FAST_DEFAULT | kMin3) : BJ_FAST_DEFAULT;
+    return (sizeof(R) == 8 && M >= 25 && M != 26)
+               ? (BJ_FAST_DEFAULT | kMin3 | ((M == 25 || M == 27 || M == 31 || M == 32) ? kOut2 : 0))
+               : (BJ_FAST_DEFAULT | ((sizeof(R) == 8 && M == 20) ? kOut2 : 0));
 }
 // Resident CTAs (of 4 warps) per SM: explicit flags, else by the registers
 // the largest order of the class needs (row in registers + ~50).
@@ -499,7 +515,8 @@ __device__ __forceinline__ void getrf_fast_tile(R *__restrict__ A, const FTask &
     // GER never touches a column after its SCAL, so those zeros are final.
     static_for<0, M>([&](auto jc) {
         constexpr int j = decltype(jc)::value;
-        redo = redo || !(fast_ok(a[j]) || (a[j] == R(0) && j < tag - 1));
+        if constexpr ((F & kOut2) != 0) redo = redo || !fast_ok_out(a[j]);
+        else redo = redo || !(fast_ok(a[j]) || (a[j] == R(0) && j < tag - 1));
     });
     // Tiles that hit a pivot ambiguity, a slow-path quotient or a failed
     // output test are redone by the safe kernel from the (still untouched)
